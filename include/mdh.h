@@ -1,0 +1,216 @@
+/*
+ * mdh.h — C-ABI of the B200 (sm_100a) MDH hot path.
+ *
+ * What this library computes (Schulze, Gorlatch, Rasch, SC-W '25, "Reduction-Aware
+ * Directive-Based Programming via Multi-Dimensional Homomorphisms"; PAPER.md = P):
+ *
+ *   out_view ∘ md_hom[I_1..I_D](f, (⊗_1..⊗_D)) ∘ inp_view          (Listing 7)
+ *
+ * i.e. for every point i of the index space [0,I_1)×…×[0,I_D) gather the input
+ * accesses x(i) = (in_b[ι_{b,a}(i)]) (inp_view), apply the scalar function
+ * y(i) = f(x(i)) (md_hom's SF), combine dimension-wise with ⊗_d — cc
+ * ("++", places by index, Listing 15) or pw(⊕) (point-wise combine into
+ * index 0, Listing 16) — and write R[j] to out_b[ω_{b,a}(j)] (out_view,
+ * P:200) with the collapsed (pw) indices equal to 0.  The definition is the
+ * footnote-2 formula; every reading of a point the paper leaves open is
+ * listed in DESIGN.md §3 (SURVEY §8(c) C-1 … C-29).
+ *
+ * Conventions (all functions):
+ *   - Every function is extern "C", returns mdh_status, never throws.
+ *   - Sizes and indices are int64_t.  Buffers are contiguous and row-major
+ *     (Listing 1 `M[i*K+k]`); transposes/strides are index functions.
+ *   - Device pointers are raw CUDA device pointers (the caller allocates them,
+ *     typically as torch tensors).  Host pointers are only taken by
+ *     mdh_execute_host and the planning calls.
+ *   - Errors: a status code; mdh_last_error() gives a thread-local message that
+ *     stays valid until the next mdh_* call on the same thread.
+ *   - No CPU fallback exists: every step of mdh_execute runs in this library's
+ *     sm_100a kernels; a library built without CUDA support does not exist.
+ */
+#ifndef MDH_H_
+#define MDH_H_
+
+#include <stddef.h>
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+#define MDH_ABI_VERSION 1
+
+#define MDH_MAX_D     10  /* MCC_Caps is 10-D (Fig 3); configs need <= 7        */
+#define MDH_MAX_RANK   8  /* buffer rank                                                */
+#define MDH_MAX_ACC    8  /* accesses per buffer (Jacobi3D: 7 to one buffer) */
+#define MDH_MAX_BUFS  32  /* PRL: 17 inputs + 3 outputs (Listing 11)         */
+#define MDH_MAX_WORLD 64  /* ranks of one multi-GPU plan                                */
+
+typedef enum {
+  MDH_OK = 0,
+  MDH_ERR_INVALID_ARG = 1,   /* null/misaligned pointer, workspace too small, bad opts  */
+  MDH_ERR_INVALID_SPEC = 2,  /* malformed: out-of-bounds access, non-injective output,  */
+                             /* size 0, f arity mismatch, declared shape too small      */
+  MDH_ERR_UNSUPPORTED = 3,   /* valid MDH but outside this build's catalog: mixed pw    */
+                             /* operators (C-3), unknown f/dtype combination, ps (NEXT)  */
+  MDH_ERR_OUT_OF_MEMORY = 4,
+  MDH_ERR_CUDA = 5,          /* a CUDA runtime/driver call or a kernel launch failed    */
+  MDH_ERR_NCCL = 6,          /* NCCL missing or an NCCL call failed                     */
+  MDH_ERR_INTERNAL = 7
+} mdh_status;
+
+/* Basic types (BSC_TYP, Listing 14; Fig 3 "Basic Type" column P:511-531). */
+typedef enum {
+  MDH_BF16 = 0,  /* bfloat16; accumulated in fp32 (reading C-13/C-15)         */
+  MDH_F32 = 1,
+  MDH_F64 = 2,
+  MDH_I32 = 3,   /* + and * wrap mod 2^32 (reading C-12)                        */
+  MDH_U32 = 4,
+  MDH_I64 = 5
+} mdh_dtype;
+
+/* Combine operators, one per dimension (combine_ops). */
+typedef enum {
+  MDH_CC = 0,              /* "++" concatenation: index set kept (Listing 15)         */
+  MDH_PW_ADD = 1,          /* pw(add)  (Listing 16 with cf = +)                      */
+  MDH_PW_MAX = 2,          /* pw(max)                                                */
+  MDH_PW_MIN = 3,          /* pw(min)                                                */
+  MDH_PW_PRL_ARGMAX = 4,   /* custom pw over the PRL record: lexicographic max of      */
+                           /* (id_measure==14, match_weight, match_id); associative and */
+                           /* commutative (reading C-19)                                */
+  MDH_PW_PRL_PAPER = 5     /* custom pw, Listing 11 prl_max literally:     */
+                           /* res = lhs if lhs.id==14 && rhs.id!=14 else rhs;           */
+                           /* associative, NOT commutative — order preserved (C-2)      */
+  /* MDH_PS_ADD: prefix-sum operator ps (Listing 17) — NEXT        */
+} mdh_combine;
+
+/* Scalar functions SF ("arbitrary but pure"); a fixed catalog here. */
+typedef enum {
+  MDH_F_MUL = 0,          /* y = x0 * x1               (f_mul); 2 accesses → 1  */
+  MDH_F_STENCIL = 1,      /* y = Σ_a w_a · x_a, w = fparams (reading C-16); n → 1        */
+  MDH_F_PRL_COMPARE = 2,  /* Fellegi–Sunter comparison of a (new, db) record pair      */
+                          /* (reading C-18): 17 accesses → (match_id i64,             */
+                          /* match_weight f64, id_measure i32); fparams = wa[8], wd[8] */
+  MDH_F_IDENTITY = 3      /* y = x0; 1 → 1                                             */
+} mdh_fn;
+
+/* An affine index function (IDX_FNC; examples P:200-206):
+ *   idx[r] = Σ_{d<D} coeff[r][d] · i_d + offset[r],   r < rank   (reading C-8)     */
+typedef struct {
+  int64_t coeff[MDH_MAX_RANK][MDH_MAX_D];
+  int64_t offset[MDH_MAX_RANK];
+} mdh_index_fn;
+
+/* A buffer and its accesses (IDF = Buffer[BSC_TYP(,shape)], Listing 12).
+ * shape all-zero ⇒ inferred as max accessed index + 1 (fn.7; reading C-9). */
+typedef struct {
+  mdh_dtype dtype;
+  int32_t rank;
+  int64_t shape[MDH_MAX_RANK];
+  int32_t n_acc;
+  mdh_index_fn acc[MDH_MAX_ACC];
+} mdh_buffer;
+
+/* The computation (Listing 7 / Listing 14). Dimension d is loop level d (C-26). */
+typedef struct {
+  int32_t D;
+  int64_t size[MDH_MAX_D];      /* I_d >= 1 (reading C-10)                          */
+  mdh_combine op[MDH_MAX_D];    /* ⊗_d                                              */
+  mdh_fn f;
+  int32_t n_fparams;
+  const double* fparams;        /* host; copied at plan time                        */
+  int32_t n_in;
+  const mdh_buffer* in;         /* host array of n_in buffers; accesses in (b,a) order */
+  int32_t n_out;
+  const mdh_buffer* out;
+} mdh_spec;
+
+#define MDH_PLAN_VIRTUAL_SHARD 0x1u  /* plan rank r of world_size on one GPU, no comm */
+#define MDH_PLAN_NO_COLLECTIVE 0x2u  /* pw shard: leave the partial result local       */
+
+typedef struct {
+  int32_t device;        /* CUDA device ordinal the plan executes on                   */
+  int32_t world_size;    /* 1 ⇒ single GPU                                             */
+  int32_t rank;
+  void* nccl_comm;       /* from mdh_comm_init, or NULL (VIRTUAL_SHARD / world 1)       */
+  int32_t shard_dim;     /* -1 ⇒ the planner chooses                                   */
+  uint32_t flags;
+  const char* tile_table;/* path of a tile table JSON; NULL ⇒ $MDH_TILE_TABLE, else the */
+                         /* table compiled into the library                             */
+  const char* force_tile;/* "key=value,…" override (like $MDH_FORCE_TILE) or NULL       */
+} mdh_plan_opts;
+
+typedef struct mdh_plan_s* mdh_plan_t;
+
+/* Validate `spec`, classify dimensions, choose a kernel template and its tiles, and
+ * (world_size > 1) rewrite the spec to this rank's sub-domain.  Host-only work: no
+ * device memory is touched except small plan-owned constants (uploaded lazily on the
+ * first execute).  Ownership: the plan copies everything it needs from `spec`.
+ * Errors: INVALID_SPEC / UNSUPPORTED as described above; INVALID_ARG for bad opts. */
+mdh_status mdh_plan(const mdh_spec* spec, const mdh_plan_opts* opts, mdh_plan_t* plan_out);
+
+/* Device workspace the caller must pass to mdh_execute (bytes, 256-B aligned start). */
+mdh_status mdh_plan_workspace_size(mdh_plan_t plan, size_t* bytes);
+
+/* The shape of input (is_output=0) or output (is_output=1) buffer `buf` as THIS rank
+ * holds it, and the global coordinates of its element 0.  world_size 1 ⇒ the global
+ * (declared or inferred) shape and zeros.  shape/global_offset: host arrays of
+ * MDH_MAX_RANK; entries >= rank are 0.  *dtype and *rank may be NULL.              */
+mdh_status mdh_plan_local_shape(mdh_plan_t plan, int32_t is_output, int32_t buf,
+                                int64_t* shape, int64_t* global_offset,
+                                int32_t* dtype, int32_t* rank);
+
+/* A JSON description of the plan (template, tiles, dimension groups, shard).  Writes
+ * at most `cap` bytes including the terminating NUL; *needed (may be NULL) gets the
+ * full length + 1. */
+mdh_status mdh_plan_describe(mdh_plan_t plan, char* json, size_t cap, size_t* needed);
+
+/* Enqueue the computation on `cuda_stream` (a cudaStream_t; NULL = legacy default).
+ *   in[b]  : device pointer of input buffer b (local shape), 16-B aligned
+ *   out[b] : device pointer of output buffer b, 16-B aligned
+ * Semantics: overwrites every output element in the image of the output index
+ * functions and leaves all others untouched ("=" not "+="; C-5, C-6);
+ * outputs need no initialisation and are never read; inputs must not alias outputs
+ * (C-27).  Asynchronous: kernel faults surface at the caller's synchronisation
+ * unless MDH_DEBUG_SYNC=1.  Deterministic: no float atomics; repeated runs are
+ * bit-identical.  With world_size > 1 and a pw shard dim the NCCL collective and
+ * the ordered local combine are enqueued on the same stream.                      */
+mdh_status mdh_execute(mdh_plan_t plan, const void* const* in, void* const* out,
+                       void* workspace, size_t workspace_bytes, void* cuda_stream);
+
+/* End-to-end variant: in/out are HOST pointers (pinned for full PCIe bandwidth).
+ * `device_scratch` (>= mdh_plan_host_scratch_size bytes) holds the device copies and
+ * the workspace.  Enqueues H2D copies, the computation and D2H copies on the stream;
+ * the caller synchronises before reading `out`.                                   */
+mdh_status mdh_plan_host_scratch_size(mdh_plan_t plan, size_t* bytes);
+mdh_status mdh_execute_host(mdh_plan_t plan, const void* const* host_in,
+                            void* const* host_out, void* device_scratch,
+                            size_t scratch_bytes, void* cuda_stream);
+
+/* Ordered ⊗-fold of S partial results of this plan (e.g. the per-rank results of a
+ * pw shard, in rank = index order): out = p_0 ⊗ p_1 ⊗ … ⊗ p_{S-1} per output element
+ * (Listing 16 applied S-1 times, lhs = lower index range).  partial_outs[s*n_out+b]
+ * is partial s of output buffer b (device, local output shape).  Only valid for
+ * plans whose reduction dims are all the same pw operator.                        */
+mdh_status mdh_combine_partials(mdh_plan_t plan, const void* const* partial_outs,
+                                int32_t S, void* const* out, void* cuda_stream);
+
+mdh_status mdh_destroy(mdh_plan_t plan);
+
+/* NCCL communicator bootstrap (NCCL is loaded with dlopen on first use).
+ * id128: 128 bytes (ncclUniqueId) produced on one rank and broadcast by the caller. */
+mdh_status mdh_comm_unique_id(void* id128);
+mdh_status mdh_comm_init(const void* id128, int32_t world, int32_t rank, int32_t device,
+                         void** comm_out);
+mdh_status mdh_comm_destroy(void* comm);
+
+const char* mdh_last_error(void);
+int32_t mdh_abi_version(void);
+
+/* Number of kernel launches the last mdh_execute/mdh_execute_host/mdh_combine_partials
+ * on this thread enqueued (for the bench's gpu_launches claim).                     */
+int32_t mdh_last_launch_count(void);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* MDH_H_ */
