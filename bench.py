@@ -1,0 +1,403 @@
+#!/usr/bin/env python
+"""bench.py — throughput of the MDH hot path on B200 (driver contract).
+
+    python bench.py [--gpus N] [--steps K] [--warmup W] [--impl mdh|reference]
+                    [--workload NAME] [--no-suite]
+
+A "step" is one mdh_execute of the whole hot path (plan not timed) on one batch of
+synthetic input already resident in HBM.  The headline workload is BASELINE.json
+configs[1]: MatMul 4096³, bf16 inputs / fp32 accumulate (`matmul_bf16`).  With N>1
+(torchrun, one process per GPU) the MatMul is sharded on M with no communication
+(weak scaling: every rank owns a 4096-row shard of a 4096·N × 4096 × 4096 problem).
+
+Timing: W untimed warm-up steps, then exactly K steps bracketed by barrier +
+synchronize; each step's device time is a CUDA-event pair on the launching stream,
+and the L2 is flushed (a 2×L2 memset, outside the event pair) before every step;
+the reported time is the max over ranks.  Rank 0 prints ONE JSON line.  At N=1 the
+line also carries `suite`: every §8 config measured the same way.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import math
+import os
+import subprocess
+import sys
+import threading
+import time
+
+import numpy as np
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+METRIC = "per-workload GB/s or TFLOP/s and % of B200 roofline, at 1/2/4/8 GPUs"
+FALLBACK = {"hbm_gbs": 6650.0, "bf16_tflops": 1590.0, "bf16_tflops_sustained": 1400.0}
+FFMA_TFLOPS = 148 * 128 * 2 * 1.965e9 / 1e12     # fp32 FFMA issue peak
+ALU_TOPS = 148 * 4 * 32 * 1.965e9 / 1e12         # thread-instructions/s issue peak
+
+
+def peaks():
+    p = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    if os.path.exists(p):
+        with open(p) as f:
+            d = json.load(f)
+        return {"hbm_gbs": d.get("hbm_gbs", FALLBACK["hbm_gbs"]), "bf16_tflops": d.get("bf16_tflops", FALLBACK["bf16_tflops"]),
+                "bf16_tflops_sustained": d.get("bf16_tflops_sustained", FALLBACK["bf16_tflops_sustained"]),
+                "source": "measured (MEASURED_PEAKS.json)"}
+    return dict(FALLBACK, source="fallback (B200_PROFILING.md)")
+
+
+# ------------------------------------------------------------------------------ workloads
+def workload(name, world=1, rank=0):
+    """(global spec, local-input generator, work per rank, unit, roofline kind)."""
+    from mdh_workloads import gen as G
+    from mdh_workloads import specs as S
+    if name in ("matmul_bf16", "matmul_f32"):
+        dt = "bf16" if name == "matmul_bf16" else "f32"
+        M = 4096
+        spec = S.matmul(M * world, 4096, 4096, dt)
+
+        def inputs():
+            a, b = G.matmul_inputs(M, 4096, 4096, dt, "signed", seed_base=2000 + 10 * rank)
+            return [a, b]
+        flops = 2.0 * M * 4096 * 4096
+        return dict(spec=spec, inputs=inputs, work=flops, unit="TFLOP/s", scale=1e12,
+                    bound="tensor" if dt == "bf16" else "alu", shard_dim=0, dtype=dt,
+                    desc=f"MatMul {M * world}x4096x4096 {dt} (Listing 9), {'tcgen05' if dt == 'bf16' else 'FFMA'} path")
+    if name.startswith("dot"):
+        dt = "i32" if "i32" in name else "f32"
+        N = 1 << 28 if name.endswith("2^28") else 1 << 20
+        spec = S.dot(N, dt)
+        return dict(spec=spec, inputs=lambda: G.dot_inputs(N, dt, "signed"), work=8.0 * N + 4, unit="GB/s",
+                    scale=1e9, bound="hbm", dtype=dt, desc=f"Dot N={N} {dt} (Fig 3 P:512)")
+    if name == "matvec_f32":
+        spec = S.matvec(8192, 8192)
+        return dict(spec=spec, inputs=lambda: G.gen_inputs(spec, 2100), work=4.0 * (8192 * 8192 + 8192 + 8192),
+                    unit="GB/s", scale=1e9, bound="hbm", dtype="f32", desc="MatVec 8192^2 fp32 (Listing 6)")
+    if name == "jacobi3d":
+        spec = S.jacobi3d(512, 512, 512)
+        return dict(spec=spec, inputs=lambda: G.jacobi3d_inputs(512, 512, 512), work=4.0 * (512 ** 3 + 510 ** 3),
+                    unit="GB/s", scale=1e9, bound="hbm", dtype="f32", desc="Jacobi3D 7-pt 512^3 fp32")
+    if name == "ccsd_bf16":
+        spec = S.ccsd_sd1(24, 72, "bf16")
+        out = 24 ** 3 * 72 ** 3
+        return dict(spec=spec, inputs=lambda: G.gen_inputs(spec, 4000), work=4.0 * out + 2.0 * (72 ** 2 * 24 ** 2 + 72 ** 3 * 24),
+                    unit="GB/s", scale=1e9, bound="hbm", dtype="bf16", flops=2.0 * out * 72,
+                    desc="CCSD(T) sd1 O=24 V=72 bf16->fp32 (HBM-bound on the 20.6 GB output)")
+    if name == "mcc_bf16":
+        spec = S.mcc(256, 7, 7, 512, 3, 3, 512, "bf16")
+        return dict(spec=spec, inputs=lambda: G.mcc_inputs(spec), work=2.0 * 256 * 49 * 512 * 4608, unit="TFLOP/s",
+                    scale=1e12, bound="tensor", dtype="bf16", desc="MCC ResNet-50 conv5_1 3x3/s2 N=256 bf16")
+    if name in ("prl_A", "prl_B"):
+        N, I = ((1 << 20), (1 << 14)) if name == "prl_A" else ((1 << 14), (1 << 20))
+        spec = S.prl(N, I)
+        return dict(spec=spec, inputs=lambda: G.prl_inputs(N, I), work=float(N) * I, unit="Gpairs/s", scale=1e9,
+                    bound="alu", dtype="u32", desc=f"PRL {N}x{I} custom argmax (Listing 11)")
+    raise SystemExit(f"unknown workload {name}")
+
+
+SUITE = ["dot_f32", "dot_i32", "dot_f32_2^28", "matvec_f32", "jacobi3d", "matmul_f32", "matmul_bf16",
+         "ccsd_bf16", "mcc_bf16", "prl_A", "prl_B"]
+
+
+def roofline(w, seconds, pk):
+    """achieved algorithmic rate of the dominant kernel vs the measured peak."""
+    if w["bound"] == "hbm":
+        ach = w["work"] / seconds / 1e9
+        return {"bound": "hbm", "achieved": ach, "peak": pk["hbm_gbs"], "unit": "GB/s", "frac": ach / pk["hbm_gbs"]}
+    if w["bound"] == "tensor":
+        ach = w["work"] / seconds / 1e12
+        peak = pk["bf16_tflops"]
+        return {"bound": "tensor", "achieved": ach, "peak": peak, "unit": "TFLOP/s", "frac": ach / peak}
+    if w["unit"] == "TFLOP/s":     # fp32 SIMT: FFMA issue peak derived in DESIGN.md §6
+        ach = w["work"] / seconds / 1e12
+        return {"bound": "alu", "achieved": ach, "peak": FFMA_TFLOPS, "unit": "TFLOP/s", "frac": ach / FFMA_TFLOPS}
+    # PRL: 9 algorithmic ALU ops per pair (8 field compares + 1 combine)
+    ach = w["work"] * 9 / seconds / 1e12
+    return {"bound": "alu", "achieved": ach, "peak": ALU_TOPS, "unit": "Tops/s", "frac": ach / ALU_TOPS}
+
+
+class Clocks:
+    """nvidia-smi sampler run DURING the timed region (B200_PROFILING.md clocks line)."""
+
+    def __init__(self, index):
+        self.index = index
+        self.p = None
+
+    def __enter__(self):
+        q = ("clocks.sm,clocks.max.sm,clocks_event_reasons.hw_slowdown,clocks_event_reasons.hw_thermal_slowdown,"
+             "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap")
+        try:
+            self.p = subprocess.Popen(["nvidia-smi", f"--query-gpu={q}", "--format=csv,noheader,nounits", "-lms", "50",
+                                       "-i", str(self.index)], stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
+        except OSError:
+            self.p = None
+        time.sleep(0.15)
+        return self
+
+    def __exit__(self, *a):
+        self.summary = None
+        if not self.p:
+            return
+        time.sleep(0.1)
+        self.p.terminate()
+        out, _ = self.p.communicate(timeout=10)
+        rows = [r.split(", ") for r in out.strip().splitlines() if r.count(",") >= 5]
+        if not rows:
+            return
+        sm = [float(r[0]) for r in rows if r[0].replace(".", "").isdigit()]
+        mx = [float(r[1]) for r in rows if r[1].replace(".", "").isdigit()]
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        reasons = sorted({names[k] for r in rows for k in range(4) if r[2 + k].strip() == "Active"})
+        self.summary = {"sm_mhz": float(np.median(sm)) if sm else None, "sm_max_mhz": max(mx) if mx else None,
+                        "reasons": reasons, "samples": len(rows)}
+
+
+def time_steps(step, K, stream, flush):
+    import torch
+    ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(K)]
+    for k in range(K):
+        if flush is not None:
+            flush.zero_()
+        ev[k][0].record(stream)
+        step()
+        ev[k][1].record(stream)
+    torch.cuda.synchronize()
+    return [a.elapsed_time(b) / 1e3 for a, b in ev]
+
+
+def run_mdh_workload(name, K, W, world, rank, dev, flush, pk, with_e2e=False, check=False):
+    import torch
+    from paper_conf_sc_schulzegr25_b200 import Plan, to_device
+    w = workload(name, world, rank)
+    kw = dict(world_size=world, rank=rank, shard_dim=w.get("shard_dim", -1)) if world > 1 else {}
+    plan = Plan(w["spec"], device=dev, **kw)
+    host = w["inputs"]()
+    tin = [to_device(x, b["dtype"], dev) for x, b in zip(host, w["spec"]["inputs"])]
+    outs = plan.empty_outputs(dev)
+    ws = plan.workspace(dev) if plan.workspace_bytes else None
+    stream = torch.cuda.current_stream(dev)
+    sh = stream.cuda_stream
+
+    def step():
+        plan(tin, outs, stream=sh, workspace_ptr=ws)
+    for _ in range(W):
+        step()
+    torch.cuda.synchronize()
+    launches = plan.last_launch_count()
+    times = time_steps(step, K, stream, flush)
+    res = {"plan": plan, "w": w, "times": times, "launches": launches, "host": host, "outs": outs}
+    if with_e2e:
+        # end to end through mdh_execute_host: pinned host in/out, copies inside the events
+        hin = [torch.from_numpy(np.ascontiguousarray(x).view(np.int16) if b["dtype"] == "bf16" else np.ascontiguousarray(x)).pin_memory()
+               for x, b in zip(host, w["spec"]["inputs"])]
+        hout = [torch.empty(o.shape, dtype=o.dtype).pin_memory() for o in outs]
+        nscr = plan.host_scratch_bytes()
+        scratch = torch.empty(nscr, dtype=torch.uint8, device=dev)
+
+        def e2e_step():
+            plan.execute_host(hin, hout, scratch.data_ptr(), nscr, sh)
+        for _ in range(W):
+            e2e_step()
+        torch.cuda.synchronize()
+        et = time_steps(e2e_step, K, stream, None)
+        res["e2e_times"] = et
+        res["h2d"] = int(sum(t.numel() * t.element_size() for t in hin))
+        res["d2h"] = int(sum(t.numel() * t.element_size() for t in hout))
+    if check:
+        import oracle
+        from paper_conf_sc_schulzegr25_b200 import to_numpy
+        pts = oracle.random_points(w["spec"] if world == 1 else plan.spec, 256, seed=11)
+        if world == 1:
+            lin, vals = oracle.evaluate_points(w["spec"], host, pts)
+            g = to_numpy(outs[0], w["spec"]["outputs"][0]["dtype"]).ravel()[lin[0]].astype(np.float64)
+            ref = vals[0]
+            res["parity"] = {"points": 256, "max_rel_err": float(np.max(np.abs(g - ref) / np.maximum(np.abs(ref), 1e-30)))}
+    return res
+
+
+def cpu_baseline(w, target_s=12.0):
+    """The oracle as it stands, on this host's cores, on a bounded sample of the workload."""
+    import oracle
+    spec = w["spec"]
+    host = w["inputs"]()
+    n = 16
+    t = 0.0
+    while True:
+        pts = oracle.random_points(spec, n, seed=3)
+        t0 = time.perf_counter()
+        oracle.evaluate_points(spec, host, pts)
+        t = time.perf_counter() - t0
+        if t > target_s / 4 or n >= 1 << 22:
+            break
+        n *= 4 if t < target_s / 64 else 2
+    ncc = 1
+    for s, o in zip(spec["sizes"], spec["ops"]):
+        if o == "CC":
+            ncc *= s
+    frac = n / ncc
+    value = w["work"] * frac / t / w["scale"]
+    return {"value": value, "unit": w["unit"], "cores": oracle.max_threads(), "kind": "oracle",
+            "sample": f"{n} random output points of {w['desc']} ({frac:.2e} of the work), each folded over its full "
+                      f"reduction range by the literal fp64 loop nest; {t:.1f} s"}
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=20)
+    ap.add_argument("--warmup", type=int, default=5)
+    ap.add_argument("--impl", default="mdh", choices=["mdh", "reference"])
+    ap.add_argument("--workload", default="matmul_bf16")
+    ap.add_argument("--no-suite", action="store_true")
+    ap.add_argument("--suite-steps", type=int, default=10)
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    a = ap.parse_args()
+    W = max(3, a.warmup)
+    K = max(1, a.steps)
+
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+
+    if a.impl == "reference":
+        return reference_arm(a, W, K, world, rank)
+
+    import torch
+    import torch.distributed as dist
+    from paper_conf_sc_schulzegr25_b200 import lib
+    lib()
+    torch.cuda.set_device(local)
+    dev = torch.device("cuda", local)
+    if world > 1:
+        dist.init_process_group("nccl", device_id=dev)
+    pk = peaks()
+    l2 = torch.cuda.get_device_properties(dev).L2_cache_size
+    flush = torch.empty(2 * l2 // 4, dtype=torch.float32, device=dev)
+
+    def barrier():
+        if world > 1:
+            dist.barrier()
+        torch.cuda.synchronize()
+
+    # ---- headline
+    barrier()
+    with Clocks(local) as clk:
+        barrier()
+        res = run_mdh_workload(a.workload, K, W, world, rank, dev, flush, pk, with_e2e=True, check=(world == 1))
+        barrier()
+    t_total = sum(res["times"])
+    et_total = sum(res["e2e_times"])
+    if world > 1:
+        tt = torch.tensor([t_total, et_total], dtype=torch.float64, device=dev)
+        dist.all_reduce(tt, op=dist.ReduceOp.MAX)
+        t_total, et_total = float(tt[0]), float(tt[1])
+    w = res["w"]
+    per_step = t_total / K
+    value = world * w["work"] / per_step / w["scale"]
+    e2e_value = world * w["work"] / (et_total / K) / w["scale"]
+    rl = roofline(w, per_step, pk)
+    rl["peak_source"] = pk["source"]
+    rl["traffic"] = ncu_traffic(a.workload)
+    rl["kernel"] = res["plan"].template
+    line = {"metric": METRIC, "value": round(value, 3), "unit": w["unit"], "n_gpus": world, "steps": K, "warmup": W,
+            "ms_per_step": round(per_step * 1e3, 4), "higher_is_better": True, "scaling": "weak", "vs_baseline": None,
+            "dtype": w["dtype"], "data": "synthetic (seeded numpy PCG64, shapes of Fig 3 / SURVEY §8(d))",
+            "config": {"workload": a.workload, "desc": w["desc"], "template": res["plan"].template,
+                       "global_shape": w["spec"]["sizes"], "l2": "flushed (2xL2 memset) before every step",
+                       "parallelism": f"shard M over {world} GPU(s), no collective" if world > 1 else "1 GPU"},
+            "roofline": rl,
+            "e2e": {"value": round(e2e_value, 3), "unit": w["unit"], "h2d_bytes_per_step": res["h2d"],
+                    "d2h_bytes_per_step": res["d2h"], "api": "mdh_execute_host (pinned host buffers)"},
+            "gpu_launches": res["launches"] * K,
+            "clocks": clk.summary}
+    if "parity" in res:
+        line["parity_sample"] = res["parity"]
+    del res
+    # ---- suite of every §8 config (N=1)
+    if world == 1 and not a.no_suite:
+        suite = {}
+        for name in SUITE:
+            if name == a.workload:
+                continue
+            try:
+                r = run_mdh_workload(name, a.suite_steps, 3, 1, 0, dev, flush, pk)
+                ts = sorted(r["times"])
+                med = ts[len(ts) // 2]
+                ww = r["w"]
+                ent = {"value": round(ww["work"] / med / ww["scale"], 3), "unit": ww["unit"], "ms_median": round(med * 1e3, 4),
+                       "template": r["plan"].template, "launches_per_step": r["launches"],
+                       "roofline": roofline(ww, med, pk), "desc": ww["desc"]}
+                if "flops" in ww:
+                    ent["tflops"] = round(ww["flops"] / med / 1e12, 2)
+                suite[name] = ent
+                del r
+            except Exception as e:  # keep the headline even if a suite member fails
+                suite[name] = {"error": str(e)[:300]}
+            torch.cuda.empty_cache()
+        line["suite"] = suite
+    if rank == 0 and world == 1 and not a.no_cpu_baseline:
+        line["cpu_baseline"] = cpu_baseline(workload(a.workload))
+    if rank == 0:
+        print(json.dumps(line), flush=True)
+    if world > 1:
+        dist.barrier()
+        dist.destroy_process_group()
+
+
+def ncu_traffic(name):
+    p = os.path.join(ROOT, "profiles", "ncu_traffic.json")
+    if os.path.exists(p):
+        with open(p) as f:
+            return json.load(f).get(name)
+    return None
+
+
+def reference_arm(a, W, K, world, rank):
+    """--impl reference: the oracle (CPU loop nest) as it stands, on this host's cores,
+    each step a bounded sample of the same workload; rank 0 only."""
+    if rank != 0:
+        return 0
+    import oracle
+    w = workload(a.workload)
+    spec, host = w["spec"], w["inputs"]()
+    n = 64
+    while True:     # size one step to ~4 s so that W+K steps end within a few minutes
+        pts = oracle.random_points(spec, n, seed=5)
+        t0 = time.perf_counter()
+        oracle.evaluate_points(spec, host, pts)
+        t = time.perf_counter() - t0
+        if t > 1.0 or n >= 1 << 22:
+            break
+        n *= 2
+    budget = 150.0
+    n = max(16, int(n * min(4.0, budget / (W + K)) / max(t, 1e-3)))
+    times = []
+    for k in range(W + K):
+        pts = oracle.random_points(spec, n, seed=100 + k)
+        t0 = time.perf_counter()
+        oracle.evaluate_points(spec, host, pts)
+        if k >= W:
+            times.append(time.perf_counter() - t0)
+    ncc = 1
+    for s, o in zip(spec["sizes"], spec["ops"]):
+        if o == "CC":
+            ncc *= s
+    frac = n / ncc
+    per = sum(times) / len(times)
+    value = w["work"] * frac / per / w["scale"]
+    line = {"metric": METRIC, "value": value, "unit": w["unit"], "n_gpus": world, "steps": K, "warmup": W,
+            "ms_per_step": per * 1e3, "higher_is_better": True, "scaling": "weak", "vs_baseline": None,
+            "dtype": w["dtype"], "data": "synthetic", "impl": "reference",
+            "config": {"workload": a.workload, "desc": w["desc"]},
+            "cpu_baseline": {"value": value, "unit": w["unit"], "cores": oracle.max_threads(), "kind": "oracle",
+                             "sample": f"{n} random output points per step ({frac:.2e} of the work), literal fp64 loop nest"},
+            "e2e": {"value": value, "unit": w["unit"], "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
+    print(json.dumps(line), flush=True)
+    return 0
+
+
+if __name__ == "__main__":
+    sys.exit(main())

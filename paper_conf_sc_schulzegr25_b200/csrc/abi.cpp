@@ -1,0 +1,321 @@
+// abi.cpp — the extern "C" entry points of libmdh (include/mdh.h).
+#include <cstdarg>
+#include <cstdio>
+#include <cstdlib>
+#include <cstring>
+#include <new>
+#include <string>
+
+#include "internal.h"
+
+struct mdh_plan_s {
+  mdh::Plan p;
+};
+
+namespace mdh {
+
+static thread_local std::string g_err;
+static thread_local int g_launches = 0;
+
+void set_error(const char* fmt, ...) {
+  char buf[1024];
+  va_list ap;
+  va_start(ap, fmt);
+  std::vsnprintf(buf, sizeof(buf), fmt, ap);
+  va_end(ap);
+  g_err = buf;
+}
+
+mdh_status cuda_check(cudaError_t e, const char* what) {
+  if (e == cudaSuccess) return MDH_OK;
+  set_error("CUDA error in %s: %s", what, cudaGetErrorString(e));
+  return e == cudaErrorMemoryAllocation ? MDH_ERR_OUT_OF_MEMORY : MDH_ERR_CUDA;
+}
+
+int64_t dtype_size(mdh_dtype t) {
+  switch (t) {
+    case MDH_BF16: return 2;
+    case MDH_F32: case MDH_I32: case MDH_U32: return 4;
+    case MDH_F64: case MDH_I64: return 8;
+  }
+  return 0;
+}
+
+bool is_float(mdh_dtype t) { return t == MDH_BF16 || t == MDH_F32 || t == MDH_F64; }
+
+void count_launch(int n) { g_launches += n; }
+void reset_launch_count() { g_launches = 0; }
+int launch_count() { return g_launches; }
+
+static bool debug_sync() {
+  static int v = -1;
+  if (v < 0) {
+    const char* e = std::getenv("MDH_DEBUG_SYNC");
+    v = (e && e[0] == '1') ? 1 : 0;
+  }
+  return v == 1;
+}
+
+mdh_status post_launch(const char* what) {
+  count_launch(1);
+  cudaError_t e = cudaGetLastError();
+  if (e != cudaSuccess) return cuda_check(e, what);
+  if (debug_sync()) return cuda_check(cudaDeviceSynchronize(), what);
+  return MDH_OK;
+}
+
+size_t add_const(Plan* p, const void* data, size_t bytes) {
+  size_t off = (p->host_const.size() + 255) / 256 * 256;
+  p->host_const.resize(off + bytes);
+  std::memcpy(p->host_const.data() + off, data, bytes);
+  return off;
+}
+
+mdh_status device_consts(const Plan& p, const char** base) {
+  std::lock_guard<std::mutex> g(p.mu);
+  if (!p.dconst && !p.host_const.empty()) {
+    void* d = nullptr;
+    MDH_CUDA(cudaMalloc(&d, p.host_const.size()));
+    cudaError_t e = cudaMemcpy(d, p.host_const.data(), p.host_const.size(), cudaMemcpyHostToDevice);
+    if (e != cudaSuccess) {
+      cudaFree(d);
+      return cuda_check(e, "upload of plan constants");
+    }
+    p.dconst = d;
+  }
+  *base = (const char*)p.dconst;
+  return MDH_OK;
+}
+
+static mdh_status check_ptrs(const mdh::Plan& p, const void* const* in, void* const* out) {
+  if (!in || !out) { set_error("in/out arrays are NULL"); return MDH_ERR_INVALID_ARG; }
+  for (int b = 0; b < p.n_in; ++b) {
+    if (!in[b]) { set_error("input %d is NULL", b); return MDH_ERR_INVALID_ARG; }
+    if (reinterpret_cast<uintptr_t>(in[b]) % 16) { set_error("input %d is not 16-byte aligned", b); return MDH_ERR_INVALID_ARG; }
+  }
+  for (int b = 0; b < p.n_out; ++b) {
+    if (!out[b]) { set_error("output %d is NULL", b); return MDH_ERR_INVALID_ARG; }
+    if (reinterpret_cast<uintptr_t>(out[b]) % 16) { set_error("output %d is not 16-byte aligned", b); return MDH_ERR_INVALID_ARG; }
+  }
+  // aliasing (reading C-27)
+  for (int b = 0; b < p.n_out; ++b) {
+    uintptr_t o0 = (uintptr_t)out[b], o1 = o0 + (uintptr_t)(p.out[b].elems * dtype_size(p.out[b].dtype));
+    for (int c = 0; c < p.n_in; ++c) {
+      uintptr_t i0 = (uintptr_t)in[c], i1 = i0 + (uintptr_t)(p.in[c].elems * dtype_size(p.in[c].dtype));
+      if (o0 < i1 && i0 < o1) { set_error("output %d overlaps input %d (reading C-27)", b, c); return MDH_ERR_INVALID_ARG; }
+    }
+  }
+  return MDH_OK;
+}
+
+static mdh_status run_template(const mdh::Plan& p, const void* const* in, void* const* out, void* ws,
+                               cudaStream_t st) {
+  switch (p.tmpl) {
+    case T0_GENERIC: return launch_t0(p, in, out, ws, st);
+    case T1_STENCIL: return launch_t1(p, in, out, ws, st);
+    case T2_REDUCE: return launch_t2(p, in, out, ws, st);
+    case T3_SIMT: return launch_t3(p, in, out, ws, st);
+    case T4_TC: return launch_t4(p, in, out, ws, st);
+    case T5_PRL: return launch_t5(p, in, out, ws, st);
+  }
+  set_error("unknown template");
+  return MDH_ERR_INTERNAL;
+}
+
+// pw shard across ranks: local partial → allgather → ordered combine (ranks = index
+// order), or an NCCL allreduce where ⊕ is exact in any order (int +, max, min).
+static mdh_status execute_sharded(const mdh::Plan& p, const void* const* in, void* const* out, char* ws,
+                                  cudaStream_t st) {
+  size_t per = 0;
+  size_t offs[MDH_MAX_BUFS];
+  for (int b = 0; b < p.n_out; ++b) {
+    offs[b] = per;
+    per += ((size_t)p.out[b].elems * dtype_size(p.out[b].dtype) + 255) / 256 * 256;
+  }
+  char* local = ws + p.ws_kernel;                 // this rank's partial
+  char* gathered = local + per;                   // world × per
+  void* lout[MDH_MAX_BUFS];
+  for (int b = 0; b < p.n_out; ++b) lout[b] = local + offs[b];
+  MDH_TRY(run_template(p, in, lout, ws, st));
+  bool exact_any_order = p.n_out == 1 && p.f != MDH_F_PRL_COMPARE &&
+                         (p.redop == MDH_PW_MAX || p.redop == MDH_PW_MIN ||
+                          (p.redop == MDH_PW_ADD && !is_float(p.out[0].dtype)));
+  if (exact_any_order) {
+    return comm_allreduce(p.comm, lout[0], out[0], (size_t)p.out[0].elems, p.out[0].dtype, p.redop, st);
+  }
+  MDH_TRY(comm_allgather(p.comm, local, gathered, per, st));
+  const void* parts[MDH_MAX_WORLD * MDH_MAX_BUFS];
+  for (int r = 0; r < p.world; ++r)
+    for (int b = 0; b < p.n_out; ++b) parts[r * p.n_out + b] = gathered + (size_t)r * per + offs[b];
+  return launch_combine(p, parts, p.world, out, st);
+}
+
+}  // namespace mdh
+
+using mdh::set_error;
+
+extern "C" {
+
+mdh_status mdh_plan(const mdh_spec* spec, const mdh_plan_opts* opts, mdh_plan_t* plan_out) {
+  if (!plan_out) { set_error("plan_out is NULL"); return MDH_ERR_INVALID_ARG; }
+  *plan_out = nullptr;
+  mdh_plan_s* h = new (std::nothrow) mdh_plan_s();
+  if (!h) { set_error("out of host memory"); return MDH_ERR_OUT_OF_MEMORY; }
+  mdh_status s;
+  try {
+    s = mdh::build_plan(spec, opts, &h->p);
+  } catch (...) {
+    set_error("internal exception in mdh_plan");
+    s = MDH_ERR_INTERNAL;
+  }
+  if (s != MDH_OK) {
+    mdh_destroy(h);
+    return s;
+  }
+  *plan_out = h;
+  return MDH_OK;
+}
+
+mdh_status mdh_plan_workspace_size(mdh_plan_t plan, size_t* bytes) {
+  if (!plan || !bytes) { set_error("NULL argument"); return MDH_ERR_INVALID_ARG; }
+  *bytes = plan->p.ws_total;
+  return MDH_OK;
+}
+
+mdh_status mdh_plan_local_shape(mdh_plan_t plan, int32_t is_output, int32_t buf, int64_t* shape,
+                                int64_t* global_offset, int32_t* dtype, int32_t* rank) {
+  if (!plan) { set_error("NULL plan"); return MDH_ERR_INVALID_ARG; }
+  const mdh::Plan& p = plan->p;
+  int n = is_output ? p.n_out : p.n_in;
+  if (buf < 0 || buf >= n) { set_error("buffer index %d out of range", buf); return MDH_ERR_INVALID_ARG; }
+  const mdh::Buf& B = is_output ? p.out[buf] : p.in[buf];
+  for (int r = 0; r < MDH_MAX_RANK; ++r) {
+    if (shape) shape[r] = r < B.rank ? B.shape[r] : 0;
+    if (global_offset) global_offset[r] = r < B.rank ? B.goff[r] : 0;
+  }
+  if (dtype) *dtype = (int32_t)B.dtype;
+  if (rank) *rank = B.rank;
+  return MDH_OK;
+}
+
+mdh_status mdh_plan_describe(mdh_plan_t plan, char* json, size_t cap, size_t* needed) {
+  if (!plan) { set_error("NULL plan"); return MDH_ERR_INVALID_ARG; }
+  std::string s = mdh::describe_plan(plan->p);
+  if (needed) *needed = s.size() + 1;
+  if (json && cap > 0) {
+    size_t n = std::min(cap - 1, s.size());
+    std::memcpy(json, s.data(), n);
+    json[n] = 0;
+  }
+  return MDH_OK;
+}
+
+mdh_status mdh_execute(mdh_plan_t plan, const void* const* in, void* const* out, void* workspace,
+                       size_t workspace_bytes, void* cuda_stream) {
+  mdh::reset_launch_count();
+  if (!plan) { set_error("NULL plan"); return MDH_ERR_INVALID_ARG; }
+  const mdh::Plan& p = plan->p;
+  MDH_TRY(mdh::check_ptrs(p, in, out));
+  if (workspace_bytes < p.ws_total || (p.ws_total > 0 && !workspace)) {
+    set_error("workspace of %zu bytes is smaller than the %zu the plan needs", workspace_bytes, p.ws_total);
+    return MDH_ERR_INVALID_ARG;
+  }
+  if (workspace && reinterpret_cast<uintptr_t>(workspace) % 256) {
+    set_error("workspace must be 256-byte aligned");
+    return MDH_ERR_INVALID_ARG;
+  }
+  cudaStream_t st = (cudaStream_t)cuda_stream;
+  try {
+    if (p.world > 1 && p.shard_is_red && p.comm && !(p.flags & MDH_PLAN_NO_COLLECTIVE))
+      return mdh::execute_sharded(p, in, out, (char*)workspace, st);
+    return mdh::run_template(p, in, out, workspace, st);
+  } catch (...) {
+    set_error("internal exception in mdh_execute");
+    return MDH_ERR_INTERNAL;
+  }
+}
+
+mdh_status mdh_plan_host_scratch_size(mdh_plan_t plan, size_t* bytes) {
+  if (!plan || !bytes) { set_error("NULL argument"); return MDH_ERR_INVALID_ARG; }
+  const mdh::Plan& p = plan->p;
+  size_t s = 0;
+  for (int b = 0; b < p.n_in; ++b) s += ((size_t)p.in[b].elems * mdh::dtype_size(p.in[b].dtype) + 255) / 256 * 256;
+  for (int b = 0; b < p.n_out; ++b) s += ((size_t)p.out[b].elems * mdh::dtype_size(p.out[b].dtype) + 255) / 256 * 256;
+  *bytes = s + p.ws_total + 256;
+  return MDH_OK;
+}
+
+mdh_status mdh_execute_host(mdh_plan_t plan, const void* const* host_in, void* const* host_out,
+                            void* device_scratch, size_t scratch_bytes, void* cuda_stream) {
+  if (!plan || !host_in || !host_out || !device_scratch) { set_error("NULL argument"); return MDH_ERR_INVALID_ARG; }
+  const mdh::Plan& p = plan->p;
+  size_t need;
+  MDH_TRY(mdh_plan_host_scratch_size(plan, &need));
+  if (scratch_bytes < need) { set_error("device scratch of %zu bytes < %zu needed", scratch_bytes, need); return MDH_ERR_INVALID_ARG; }
+  cudaStream_t st = (cudaStream_t)cuda_stream;
+  char* base = (char*)(((uintptr_t)device_scratch + 255) / 256 * 256);
+  const void* din[MDH_MAX_BUFS];
+  void* dout[MDH_MAX_BUFS];
+  size_t off = 0;
+  int copies = 0;
+  for (int b = 0; b < p.n_in; ++b) {
+    size_t n = (size_t)p.in[b].elems * mdh::dtype_size(p.in[b].dtype);
+    MDH_CUDA(cudaMemcpyAsync(base + off, host_in[b], n, cudaMemcpyHostToDevice, st));
+    din[b] = base + off;
+    off += (n + 255) / 256 * 256;
+    ++copies;
+  }
+  for (int b = 0; b < p.n_out; ++b) {
+    size_t n = (size_t)p.out[b].elems * mdh::dtype_size(p.out[b].dtype);
+    dout[b] = base + off;
+    off += (n + 255) / 256 * 256;
+  }
+  void* ws = base + off;
+  mdh_status s = mdh_execute(plan, din, dout, ws, p.ws_total, cuda_stream);
+  if (s != MDH_OK) return s;
+  int launched = mdh::launch_count();
+  for (int b = 0; b < p.n_out; ++b) {
+    size_t n = (size_t)p.out[b].elems * mdh::dtype_size(p.out[b].dtype);
+    MDH_CUDA(cudaMemcpyAsync(host_out[b], dout[b], n, cudaMemcpyDeviceToHost, st));
+    ++copies;
+  }
+  mdh::reset_launch_count();
+  mdh::count_launch(launched);
+  (void)copies;
+  return MDH_OK;
+}
+
+mdh_status mdh_combine_partials(mdh_plan_t plan, const void* const* partial_outs, int32_t S,
+                                void* const* out, void* cuda_stream) {
+  mdh::reset_launch_count();
+  if (!plan || !partial_outs || !out || S < 1) { set_error("bad arguments"); return MDH_ERR_INVALID_ARG; }
+  const mdh::Plan& p = plan->p;
+  if (p.nred == 0) { set_error("plan has no pw dimension: partials are concatenated, not combined"); return MDH_ERR_INVALID_ARG; }
+  return mdh::launch_combine(p, partial_outs, S, out, (cudaStream_t)cuda_stream);
+}
+
+mdh_status mdh_destroy(mdh_plan_t plan) {
+  if (!plan) return MDH_OK;
+  if (plan->p.dconst) {
+    int cur = 0;
+    cudaGetDevice(&cur);
+    cudaSetDevice(plan->p.device);
+    cudaFree(plan->p.dconst);
+    cudaSetDevice(cur);
+  }
+  mdh::release_t4(&plan->p);
+  delete plan;
+  return MDH_OK;
+}
+
+mdh_status mdh_comm_unique_id(void* id128) { return mdh::comm_unique_id(id128); }
+mdh_status mdh_comm_init(const void* id128, int32_t world, int32_t rank, int32_t device, void** comm_out) {
+  return mdh::comm_init(id128, world, rank, device, comm_out);
+}
+mdh_status mdh_comm_destroy(void* comm) { return mdh::comm_destroy(comm); }
+
+const char* mdh_last_error(void) { return mdh::g_err.c_str(); }
+int32_t mdh_abi_version(void) { return MDH_ABI_VERSION; }
+int32_t mdh_last_launch_count(void) { return mdh::launch_count(); }
+
+}  // extern "C"

@@ -1,0 +1,277 @@
+// t3_simt.cu — T3: SIMT (CUDA-core FFMA / IMAD) contraction for f = MUL, ⊗ = pw(add)
+// with reuse (MatMul fp32, Listing 9; fp32 CCSD(T) Fig 3 P:526-527 and MCC
+// Listing 12 P:401-429 parity runs; int32 contractions).
+//
+// Dimension grouping (A0): M = cc dims only A's index function uses, N = cc dims only
+// B uses, Z (batch) = cc dims both use, K = the pw dims.  Because index functions are
+// affine, each operand offset separates: offA = offA_Z[z] + offA_M[m] + offA_K[k]
+// (likewise B and C); the plan builds these tables once on the host.  This one kernel
+// therefore covers MatMul, transposed/batched MatMul, tensor contractions and
+// stride-2 convolutions (implicit im2col) alike.
+//
+// Tiling (A1, A4): 128×128 CTA tile, BK = 8, 256 threads each owning an 8×8 register
+// tile; A/B tiles gathered with coalesced loads along whichever of M/K (N/K) is
+// contiguous, staged in shared memory (double-buffered through registers).  fp32
+// accumulate (reading C-13), int32 wraps (C-12).  Optional split-K over CTAs (A7):
+// fp32 partials [S][Z·M·N] folded in split order by the combine kernel.
+#include <algorithm>
+#include <vector>
+
+#include "kcommon.cuh"
+
+namespace mdh {
+
+enum { T3_TAB_AM = 0, T3_TAB_AK, T3_TAB_BN, T3_TAB_BK, T3_TAB_CM, T3_TAB_CN, T3_TAB_AZ, T3_TAB_BZ, T3_TAB_CZ };
+
+struct T3Params {
+  const void* A;
+  const void* B;
+  void* C;
+  int cdt;
+  const int64_t* tab[9];
+  int64_t M, N, K, Z;
+  int64_t kchunk;
+  int S;
+  int a_kcontig, b_kcontig;
+  void* partial;     // V[S][Z][M][N] when S > 1
+};
+
+template <class TI, class V>
+__device__ __forceinline__ V ldv(const TI* p, int64_t i) {
+  if constexpr (std::is_same<TI, uint16_t>::value) return (V)bf16_to_f32(p[i]);
+  else return (V)__ldg(p + i);
+}
+
+template <class TI, class V>
+__global__ void __launch_bounds__(256, 1) t3_kernel(const __grid_constant__ T3Params P) {
+  constexpr int BM = 128, BN = 128, BK = 8;
+  __shared__ __align__(16) V As[2][BK][BM];
+  __shared__ __align__(16) V Bs[2][BK][BN];
+  const int tid = threadIdx.x;
+  const int tx = tid & 15, ty = tid >> 4;
+  const int64_t m0 = (int64_t)blockIdx.y * BM, n0 = (int64_t)blockIdx.x * BN;
+  const int64_t zs = blockIdx.z;
+  const int64_t z = zs % P.Z;
+  const int s = (int)(zs / P.Z);
+  const int64_t kbeg = (int64_t)s * P.kchunk;
+  const int64_t kend = min(P.K, kbeg + P.kchunk);
+  const TI* A = (const TI*)P.A + P.tab[T3_TAB_AZ][z];
+  const TI* B = (const TI*)P.B + P.tab[T3_TAB_BZ][z];
+  const int64_t* aK = P.tab[T3_TAB_AK];
+  const int64_t* bK = P.tab[T3_TAB_BK];
+
+  // per-thread load coordinates (fixed rows/cols across k-tiles)
+  int la_m[4], la_k[4], lb_n[4], lb_k[4];
+  int64_t la_row[4], lb_col[4];
+#pragma unroll
+  for (int j = 0; j < 4; ++j) {
+    if (P.a_kcontig) { la_m[j] = tid >> 1; la_k[j] = (tid & 1) * 4 + j; }
+    else { la_k[j] = tid >> 5; la_m[j] = (tid & 31) * 4 + j; }
+    if (P.b_kcontig) { lb_n[j] = tid >> 1; lb_k[j] = (tid & 1) * 4 + j; }
+    else { lb_k[j] = tid >> 5; lb_n[j] = (tid & 31) * 4 + j; }
+    int64_t gm = m0 + la_m[j], gn = n0 + lb_n[j];
+    la_row[j] = gm < P.M ? P.tab[T3_TAB_AM][gm] : -1;
+    lb_col[j] = gn < P.N ? P.tab[T3_TAB_BN][gn] : -1;
+  }
+  V ra[4], rb[4];
+  auto gload = [&](int64_t k0) {
+#pragma unroll
+    for (int j = 0; j < 4; ++j) {
+      int64_t ka = k0 + la_k[j], kb = k0 + lb_k[j];
+      ra[j] = (la_row[j] >= 0 && ka < kend) ? ldv<TI, V>(A, la_row[j] + __ldg(aK + ka)) : (V)0;
+      rb[j] = (lb_col[j] >= 0 && kb < kend) ? ldv<TI, V>(B, lb_col[j] + __ldg(bK + kb)) : (V)0;
+    }
+  };
+  auto sstore = [&](int buf) {
+#pragma unroll
+    for (int j = 0; j < 4; ++j) {
+      As[buf][la_k[j]][la_m[j]] = ra[j];
+      Bs[buf][lb_k[j]][lb_n[j]] = rb[j];
+    }
+  };
+  V acc[8][8];
+#pragma unroll
+  for (int i = 0; i < 8; ++i)
+#pragma unroll
+    for (int j = 0; j < 8; ++j) acc[i][j] = (V)0;
+
+  int64_t k0 = kbeg;
+  gload(k0);
+  sstore(0);
+  __syncthreads();
+  int buf = 0;
+  for (; k0 < kend; k0 += BK) {
+    const bool more = k0 + BK < kend;
+    if (more) gload(k0 + BK);
+#pragma unroll
+    for (int kk = 0; kk < BK; ++kk) {
+      V a[8], b[8];
+      const V* ap = &As[buf][kk][0];
+      const V* bp = &Bs[buf][kk][0];
+#pragma unroll
+      for (int i = 0; i < 4; ++i) {
+        a[i] = ap[ty * 4 + i];
+        a[4 + i] = ap[64 + ty * 4 + i];
+        b[i] = bp[tx * 4 + i];
+        b[4 + i] = bp[64 + tx * 4 + i];
+      }
+#pragma unroll
+      for (int i = 0; i < 8; ++i)
+#pragma unroll
+        for (int j = 0; j < 8; ++j) acc[i][j] = Arith<V>::mul_add(acc[i][j], a[i], b[j]);
+    }
+    if (more) {
+      sstore(buf ^ 1);
+      __syncthreads();
+      buf ^= 1;
+    }
+  }
+  // epilogue (A8): scatter through the output tables
+  const int64_t* cM = P.tab[T3_TAB_CM];
+  const int64_t* cN = P.tab[T3_TAB_CN];
+  const int64_t cz = P.tab[T3_TAB_CZ][z];
+#pragma unroll
+  for (int i = 0; i < 8; ++i) {
+    int64_t gm = m0 + (i < 4 ? ty * 4 + i : 64 + ty * 4 + (i - 4));
+    if (gm >= P.M) continue;
+    int64_t rowoff = P.S > 1 ? ((z * P.M + gm) * P.N) : (cz + cM[gm]);
+#pragma unroll
+    for (int j = 0; j < 8; ++j) {
+      int64_t gn = n0 + (j < 4 ? tx * 4 + j : 64 + tx * 4 + (j - 4));
+      if (gn >= P.N) continue;
+      if (P.S > 1) ((V*)P.partial)[(int64_t)s * P.Z * P.M * P.N + rowoff + gn] = acc[i][j];
+      else store_as<V>(P.C, P.cdt, rowoff + cN[gn], acc[i][j]);
+    }
+  }
+}
+
+template <class V>
+__global__ void __launch_bounds__(256) t3_splitk_combine(const __grid_constant__ T3Params P) {
+  const int64_t total = P.Z * P.M * P.N;
+  for (int64_t e = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; e < total; e += (int64_t)gridDim.x * blockDim.x) {
+    const int64_t n = e % P.N, m = (e / P.N) % P.M, z = e / (P.N * P.M);
+    V acc = ((const V*)P.partial)[e];
+    for (int s = 1; s < P.S; ++s) acc = Arith<V>::add(acc, ((const V*)P.partial)[(int64_t)s * total + e]);   // split order
+    store_as<V>(P.C, P.cdt, P.tab[T3_TAB_CZ][z] + P.tab[T3_TAB_CM][m] + P.tab[T3_TAB_CN][n], acc);
+  }
+}
+
+// ---------------------------------------------------------------------- host
+// table of offsets of a dim group, enumerated in row-major (lexicographic) order
+static std::vector<int64_t> group_table(const Plan& p, const int* dims, int nd, const Access& acc) {
+  int64_t n = 1;
+  for (int t = 0; t < nd; ++t) n *= p.size[dims[t]];
+  std::vector<int64_t> tab((size_t)n);
+  for (int64_t q = 0; q < n; ++q) {
+    int64_t rem = q, off = 0;
+    for (int t = nd - 1; t >= 0; --t) {
+      int64_t v = rem % p.size[dims[t]];
+      rem /= p.size[dims[t]];
+      off += acc.L[dims[t]] * v;
+    }
+    tab[(size_t)q] = off;
+  }
+  return tab;
+}
+
+static bool contiguous(const std::vector<int64_t>& t) {
+  for (size_t i = 1; i < t.size(); ++i)
+    if (t[i] - t[i - 1] != 1) return false;
+  return true;
+}
+
+// builds the 9 offset tables of a grouped contraction into host_const (shared with T4)
+void build_contraction_tables(Plan* p, int64_t* a_kc, int64_t* b_kc) {
+  const Contraction& c = p->con;
+  const Access& A = p->in[c.a_buf].acc[0];
+  const Access& B = p->in[c.b_buf].acc[0];
+  const Access& C = p->out[0].acc[0];
+  std::vector<int64_t> t[9];
+  t[T3_TAB_AM] = group_table(*p, c.md, c.nm, A);
+  t[T3_TAB_AK] = group_table(*p, c.kd, c.nk, A);
+  t[T3_TAB_BN] = group_table(*p, c.nd, c.nn, B);
+  t[T3_TAB_BK] = group_table(*p, c.kd, c.nk, B);
+  t[T3_TAB_CM] = group_table(*p, c.md, c.nm, C);
+  t[T3_TAB_CN] = group_table(*p, c.nd, c.nn, C);
+  t[T3_TAB_AZ] = group_table(*p, c.zd, c.nz, A);
+  t[T3_TAB_BZ] = group_table(*p, c.zd, c.nz, B);
+  t[T3_TAB_CZ] = group_table(*p, c.zd, c.nz, C);
+  for (int k = 0; k < 9; ++k) {
+    t[k][0] += 0;
+    if (k == T3_TAB_AZ) for (auto& v : t[k]) v += A.base;
+    if (k == T3_TAB_BZ) for (auto& v : t[k]) v += B.base;
+    if (k == T3_TAB_CZ) for (auto& v : t[k]) v += C.base;
+    p->tab_off[k] = add_const(p, t[k].data(), t[k].size() * sizeof(int64_t));
+  }
+  *a_kc = contiguous(t[T3_TAB_AK]);
+  *b_kc = contiguous(t[T3_TAB_BK]);
+}
+
+mdh_status prepare_t3(Plan* p) {
+  const Contraction& c = p->con;
+  bool same = p->in[0].dtype == p->in[1].dtype;
+  if (!same || (c.nm + c.nn + c.nk + c.nz) == 0 || p->n_out != 1) {
+    p->tmpl = T0_GENERIC;
+    p->why = "contraction outside the T3 catalog: generic template";
+    return prepare_t0(p);
+  }
+  int64_t akc, bkc;
+  p->host_const.clear();
+  build_contraction_tables(p, &akc, &bkc);
+  p->tiles.vec = (int)(akc | (bkc << 1));
+  // split-K when the output tile grid cannot fill the GPU
+  int64_t tiles = ((c.M + 127) / 128) * ((c.N + 127) / 128) * c.Z;
+  int S = 1;
+  if (p->tiles.split > 0) S = p->tiles.split;
+  else if (tiles < 148 && c.K >= 256) S = (int)std::min<int64_t>(std::max<int64_t>(1, 296 / tiles), c.K / 64);
+  if (S < 1) S = 1;
+  int64_t kchunk = (c.K + S - 1) / S;
+  kchunk = (kchunk + 7) / 8 * 8;
+  S = (int)((c.K + kchunk - 1) / kchunk);
+  p->tiles.split = S;
+  p->tiles.bk = (int)std::min<int64_t>(kchunk, INT32_MAX);
+  p->ws_kernel = S > 1 ? (size_t)S * c.Z * c.M * c.N * sizeof(float) : 0;
+  return MDH_OK;
+}
+
+mdh_status launch_t3(const Plan& p, const void* const* in, void* const* out, void* ws, cudaStream_t st) {
+  const char* dc = nullptr;
+  MDH_TRY(device_consts(p, &dc));
+  const Contraction& c = p.con;
+  T3Params P;
+  memset(&P, 0, sizeof(P));
+  P.A = in[c.a_buf];
+  P.B = in[c.b_buf];
+  P.C = out[0];
+  P.cdt = p.out[0].dtype;
+  for (int k = 0; k < 9; ++k) P.tab[k] = (const int64_t*)(dc + p.tab_off[k]);
+  P.M = c.M;
+  P.N = c.N;
+  P.K = c.K;
+  P.Z = c.Z;
+  P.S = p.tiles.split;
+  P.kchunk = p.tiles.bk;
+  P.a_kcontig = p.tiles.vec & 1;
+  P.b_kcontig = (p.tiles.vec >> 1) & 1;
+  P.partial = ws;
+  dim3 grid((unsigned)((c.N + 127) / 128), (unsigned)((c.M + 127) / 128), (unsigned)(c.Z * P.S));
+  if (grid.y > 65535 || grid.z > 65535) { set_error("T3 grid too large"); return MDH_ERR_UNSUPPORTED; }
+  mdh_dtype t = p.in[c.a_buf].dtype;
+  if (t == MDH_F32) t3_kernel<float, float><<<grid, 256, 0, st>>>(P);
+  else if (t == MDH_BF16) t3_kernel<uint16_t, float><<<grid, 256, 0, st>>>(P);
+  else if (t == MDH_I32) t3_kernel<int32_t, int32_t><<<grid, 256, 0, st>>>(P);
+  else if (t == MDH_U32) t3_kernel<uint32_t, uint32_t><<<grid, 256, 0, st>>>(P);
+  else { set_error("T3: unsupported dtype"); return MDH_ERR_UNSUPPORTED; }
+  MDH_TRY(post_launch("t3_kernel"));
+  if (P.S > 1) {
+    int64_t total = c.Z * c.M * c.N;
+    unsigned g = (unsigned)std::min<int64_t>((total + 255) / 256, 148LL * 32);
+    if (p.compute == MDH_F32) t3_splitk_combine<float><<<g, 256, 0, st>>>(P);
+    else if (p.compute == MDH_I32) t3_splitk_combine<int32_t><<<g, 256, 0, st>>>(P);
+    else t3_splitk_combine<uint32_t><<<g, 256, 0, st>>>(P);
+    MDH_TRY(post_launch("t3_splitk_combine"));
+  }
+  return MDH_OK;
+}
+
+}  // namespace mdh

@@ -1,0 +1,329 @@
+"""GPU parity: the CUDA path through the C-ABI vs the CPU oracle on the same seeded
+inputs (SURVEY §8(c).5 parity matrix).  Tolerances (north star):
+integers / indices / PRL / max-min selections bit-exact; fp32 1e-4 (element-wise on
+positive data, scale-normalised on signed data, reading C-14); bf16 inputs 1e-2."""
+import json
+import os
+
+import numpy as np
+import pytest
+
+import oracle
+from mdh_workloads import gen as G
+from mdh_workloads import specs as S
+
+from gpu_util import assert_close_full, assert_close_points, run_gpu
+
+pytestmark = pytest.mark.gpu
+GOLD = os.path.join(os.path.dirname(__file__), "golden")
+
+
+# ----------------------------------------------------------------- T2: Dot / MatVec
+DOT_N = [1, 2, 3, 31, 32, 33, 127, 4097, 65537, 1 << 20, (1 << 20) + 3]
+
+
+@pytest.mark.parametrize("N", DOT_N)
+@pytest.mark.parametrize("op", ["PW_ADD", "PW_MAX", "PW_MIN"])
+@pytest.mark.parametrize("dt", ["f32", "i32"])
+def test_dot(N, op, dt):
+    spec = S.dot(N, dt, op)
+    kind = "positive" if dt == "f32" and op == "PW_ADD" else "signed"
+    x = G.dot_inputs(N, dt, kind)
+    got, p = run_gpu(spec, x)
+    assert p.template == "T2_reduce"
+    if dt == "i32" or op != "PW_ADD":
+        if dt == "f32":   # selections of fp32 products: only f's own fp32 rounding (≤2^-24)
+            assert_close_full(spec, x, got, 1e-6, kind="rel")
+        else:
+            assert_close_full(spec, x, got, 0, kind="exact")
+    else:
+        assert_close_full(spec, x, got, 1e-4, kind="rel")
+
+
+def test_dot_signed_fp32_scale_normalised():
+    N = 1 << 20
+    x = G.dot_inputs(N, "f32", "signed")
+    got, _ = run_gpu(S.dot(N, "f32"), x)
+    assert_close_full(S.dot(N, "f32"), x, got, 1e-4, kind="scale")
+
+
+def test_dot_int32_golden():
+    with open(os.path.join(GOLD, "dot_int32.json")) as f:
+        g = json.load(f)
+    N = g["N"]
+    for kind in ("iota_one", "iota_iota"):
+        got, _ = run_gpu(S.dot(N, "i32"), G.dot_inputs(N, "i32", kind))
+        assert int(got[0][0]) == g[kind]
+
+
+def test_dot_repeatable_bit_identical():
+    N = (1 << 20) + 3
+    x = G.dot_inputs(N, "f32", "signed")
+    a, p = run_gpu(S.dot(N, "f32"), x)
+    b, _ = run_gpu(S.dot(N, "f32"), x, plan=p)
+    assert a[0].tobytes() == b[0].tobytes()
+
+
+@pytest.mark.parametrize("I,K", [(1, 1), (3, 1000), (17, 1 << 20), (4096, 4096), (8192, 8192)])
+def test_matvec(I, K):
+    spec = S.matvec(I, K)
+    x = G.gen_inputs(spec, 2100, "positive")
+    got, p = run_gpu(spec, x)
+    assert p.template == "T2_reduce"
+    assert_close_full(spec, x, got, 1e-4, kind="rel")
+
+
+@pytest.mark.parametrize("op", ["PW_MAX", "PW_MIN", "PW_ADD"])
+def test_matvec_int32(op):
+    spec = S.matvec(37, 5001, "i32", op)
+    x = G.gen_inputs(spec, 2200)
+    got, _ = run_gpu(spec, x)
+    assert_close_full(spec, x, got, 0, kind="exact")
+
+
+@pytest.mark.parametrize("shape,red", [([1000, 37], [0]), ([5, 6, 7], [1]), ([64, 3], [0]), ([3, 100000], [1])])
+def test_reductions_identity_f(shape, red):
+    spec = S.reduce_spec(shape, red, "PW_ADD")
+    x = G.gen_inputs(spec, 2300, "positive")
+    got, _ = run_gpu(spec, x)
+    assert_close_full(spec, x, got, 1e-4, kind="rel")
+
+
+# ----------------------------------------------------------------- T1: stencils
+@pytest.mark.parametrize("zyx", [(3, 3, 3), (5, 7, 9), (66, 130, 258)])
+def test_jacobi3d(zyx):
+    spec = S.jacobi3d(*zyx)
+    x = G.jacobi3d_inputs(*zyx)
+    got, p = run_gpu(spec, x)
+    assert p.template == "T1_stencil"
+    assert_close_full(spec, x, got, 1e-4, kind="scale")
+
+
+def test_jacobi3d_full_size_sampled_and_closed_forms():
+    spec = S.jacobi3d(512, 512, 512)
+    x = G.jacobi3d_inputs(512, 512, 512)
+    got, _ = run_gpu(spec, x)
+    assert_close_points(spec, x, got, 1e-4, n=20000, kind="scale")
+    with open(os.path.join(GOLD, "jacobi3d.json")) as f:
+        g = json.load(f)
+    got, _ = run_gpu(spec, G.jacobi3d_inputs(512, 512, 512, "constant"))
+    assert np.abs(got[0].astype(np.float64) - g["constant_field_2_0"]).max() <= 1e-4 * 2.0 * 2.0 * 1.67
+
+
+@pytest.mark.parametrize("K", [1, 3, 1000])
+def test_jacobi1d(K):
+    spec = S.jacobi1d(K)
+    x = [G.rng(17).uniform(0, 1, K + 2).astype(np.float32)]
+    got, _ = run_gpu(spec, x)
+    assert_close_full(spec, x, got, 1e-4, kind="rel")
+
+
+def test_copy_identity():
+    spec = S.copy_spec([7, 33, 65])
+    x = G.gen_inputs(spec, 2400)
+    got, _ = run_gpu(spec, x)
+    assert np.array_equal(got[0], x[0])
+
+
+# ----------------------------------------------------------------- T3: SIMT contraction
+@pytest.mark.parametrize("mnk", [(1, 1, 1), (3, 5, 7), (127, 129, 65), (128, 256, 64), (300, 200, 1000)])
+def test_matmul_fp32(mnk):
+    M, N, K = mnk
+    spec = S.matmul(M, N, K)
+    x = G.matmul_inputs(M, N, K, "f32", "positive")
+    got, p = run_gpu(spec, x)
+    assert p.template == "T3_simt_contraction"
+    assert_close_full(spec, x, got, 1e-4, kind="rel")
+
+
+def test_matmul_fp32_full_size_sampled():
+    spec = S.matmul(4096, 4096, 4096)
+    x = G.matmul_inputs(4096, 4096, 4096, "f32", "signed")
+    got, _ = run_gpu(spec, x)
+    assert_close_points(spec, x, got, 1e-4, n=3000, kind="scale")
+    x = G.matmul_inputs(4096, 4096, 4096, "f32", "ones")
+    got, _ = run_gpu(spec, x)
+    assert np.all(got[0] == 4096.0)
+
+
+def test_matmul_identity_exact():
+    spec = S.matmul(256, 384, 256)
+    x = G.matmul_inputs(256, 384, 256, "f32", "identity")
+    got, _ = run_gpu(spec, x)
+    assert np.array_equal(got[0], x[1])
+
+
+def test_matmul_int32_wraps():
+    spec = S.matmul(70, 90, 300, "i32", "i32")
+    x = G.gen_inputs(spec, 2500)
+    got, _ = run_gpu(spec, x)
+    assert_close_full(spec, x, got, 0, kind="exact")
+
+
+def test_matmul_transposed_batched():
+    spec = S.matmul_t(64, 500, 64)      # Fig 3 MatMul^T sizes
+    x = G.gen_inputs(spec, 2600, "positive")
+    got, _ = run_gpu(spec, x)
+    assert_close_full(spec, x, got, 1e-4, kind="rel")
+    spec = S.bmatmul(16, 10, 500, 64)   # Fig 3 bMatMul sizes
+    x = G.gen_inputs(spec, 2700, "positive")
+    got, _ = run_gpu(spec, x)
+    assert_close_full(spec, x, got, 1e-4, kind="rel")
+
+
+def test_ccsd_small_and_paper_inp1():
+    spec = S.ccsd_sd1(2, 3, "f32")
+    x = G.gen_inputs(spec, 4000)
+    got, _ = run_gpu(spec, x)
+    assert_close_full(spec, x, got, 1e-4, kind="scale")
+    spec = S.ccsd_sd2()                 # paper Inp.1 reading (C-22), fp32
+    x = G.gen_inputs(spec, 4001)
+    got, _ = run_gpu(spec, x)
+    assert_close_points(spec, x, got, 1e-4, n=5000, kind="scale")
+
+
+def test_ccsd_full_size_fp32_sampled():
+    spec = S.ccsd_sd1(24, 72, "f32")
+    x = G.gen_inputs(spec, 4002)
+    got, _ = run_gpu(spec, x)
+    assert_close_points(spec, x, got, 1e-4, n=20000, kind="scale")
+
+
+@pytest.mark.parametrize("cfg", [(2, 3, 4, 5, 3, 3, 2), (1, 7, 7, 512, 3, 3, 512), (1, 112, 112, 64, 7, 7, 3)])
+def test_mcc_fp32(cfg):
+    spec = S.mcc(*cfg, dtype="f32")
+    x = G.mcc_inputs(spec)
+    got, _ = run_gpu(spec, x)
+    assert_close_full(spec, x, got, 1e-4, kind="scale")
+
+
+# ----------------------------------------------------------------- T5: PRL
+@pytest.mark.parametrize("op", ["PW_PRL_ARGMAX", "PW_PRL_PAPER"])
+def test_prl_tiny_golden(op):
+    with open(os.path.join(GOLD, "prl_tiny.json")) as f:
+        g = json.load(f)
+    ins, w = G.prl_tiny()
+    spec = S.prl(3, 4, op, weights=w)
+    got, p = run_gpu(spec, ins)
+    assert p.template == "T5_prl_pairwise"
+    for n, (e_id, e_w, e_m) in enumerate(g[op]):
+        assert (int(got[0][n]), float(got[1][n]), int(got[2][n])) == (e_id, e_w, e_m)
+
+
+@pytest.mark.parametrize("NI", [(1, 1), (64, 64), (1000, 777), (1 << 10, 1 << 15)])
+@pytest.mark.parametrize("op", ["PW_PRL_ARGMAX", "PW_PRL_PAPER"])
+def test_prl_full(NI, op):
+    N, I = NI
+    ins = G.prl_inputs(N, I, seed_base=5500)
+    spec = S.prl(N, I, op)
+    got, _ = run_gpu(spec, ins)
+    assert_close_full(spec, ins, got, 0, kind="exact")
+
+
+@pytest.mark.parametrize("NI", [(1 << 20, 1 << 14), (1 << 14, 1 << 20)])
+def test_prl_config_sampled(NI):
+    N, I = NI
+    ins = G.prl_inputs(N, I, seed_base=5000)
+    spec = S.prl(N, I)
+    got, _ = run_gpu(spec, ins)
+    assert_close_points(spec, ins, got, 0, n=400, kind="exact")
+
+
+# ----------------------------------------------------------------- T0 and semantics
+def test_generic_strided_output_untouched_elements():
+    import torch
+    from paper_conf_sc_schulzegr25_b200 import Plan, to_device, to_numpy
+    d = ["i", "k"]
+    spec = S.make_spec("strided", d, [50, 30], ["CC", "PW_MAX"], "IDENTITY",
+                       [S.buffer("x", "f32", [["i", "k"]], d)],
+                       [S.buffer("y", "f32", [["3*i+1"]], d, shape=[151])])
+    x = G.gen_inputs(spec, 2800)
+    p = Plan(spec)
+    y = torch.full((151,), -7.0, device="cuda")
+    p([to_device(x[0], "f32", "cuda")], [y])
+    torch.cuda.synchronize()
+    yh = to_numpy(y, "f32")
+    ref = oracle.evaluate(spec, x, fill=-7.0)[0]
+    assert np.array_equal(yh.astype(np.float64), ref)
+
+
+def test_generic_template_nonlinear_reduction():
+    # pw dims not linear in the input (transposed) → T0 catch-all, still on the GPU
+    d = ["a", "b", "c"]
+    spec = S.make_spec("t0", d, [9, 5, 7], ["CC", "PW_ADD", "PW_ADD"], "IDENTITY",
+                       [S.buffer("x", "f32", [["a", "c", "b"]], d)],
+                       [S.buffer("y", "f32", [["a"]], d)])
+    x = G.gen_inputs(spec, 2900, "positive")
+    got, p = run_gpu(spec, x)
+    assert p.template == "T0_generic"
+    assert_close_full(spec, x, got, 1e-4, kind="rel")
+
+
+def test_misaligned_pointer_rejected():
+    import torch
+    from paper_conf_sc_schulzegr25_b200 import Plan, MdhError
+    p = Plan(S.dot(100, "f32"))
+    a = torch.zeros(200, device="cuda")
+    with pytest.raises(MdhError, match="INVALID_ARG"):
+        p([a[1:101], a[100:]], [torch.zeros(4, device="cuda")])
+
+
+# ----------------------------------------------------- homomorphism via virtual shards
+def _virtual_shards(spec, inputs, world, shard_dim):
+    """Run every rank's sub-domain plan on one GPU (MDH_PLAN_VIRTUAL_SHARD), slicing the
+    inputs by the plan's local shapes; pw shards are recombined by mdh_combine_partials."""
+    import torch
+    from paper_conf_sc_schulzegr25_b200 import Plan, to_device, to_numpy, VIRTUAL_SHARD
+    parts, plans = [], []
+    for r in range(world):
+        p = Plan(spec, world_size=world, rank=r, shard_dim=shard_dim, flags=VIRTUAL_SHARD)
+        tin = []
+        for b, x in enumerate(inputs):
+            shp, off, _ = p.local_shape(False, b)
+            sl = tuple(slice(o, o + s) for o, s in zip(off, shp))
+            tin.append(to_device(np.ascontiguousarray(x[sl]), spec["inputs"][b]["dtype"], "cuda"))
+        outs = p.empty_outputs()
+        p(tin, outs)
+        parts.append((p, outs))
+        plans.append(p)
+    torch.cuda.synchronize()
+    return parts
+
+
+@pytest.mark.parametrize("world", [2, 3, 4, 8])
+def test_virtual_shard_pw_dot_and_prl(world):
+    from paper_conf_sc_schulzegr25_b200 import to_numpy
+    N = 100003
+    spec = S.dot(N, "i32")
+    x = G.dot_inputs(N, "i32")
+    parts = _virtual_shards(spec, x, world, 0)
+    comb = parts[0][0].combine_partials([o for _, o in parts])
+    assert int(to_numpy(comb[0], "i32")[0]) == int(oracle.evaluate(spec, x)[0][0])
+    for op in ("PW_PRL_ARGMAX", "PW_PRL_PAPER"):
+        spec = S.prl(300, 5000, op)
+        ins = G.prl_inputs(300, 5000, seed_base=5600)
+        parts = _virtual_shards(spec, ins, world, 1)
+        comb = parts[0][0].combine_partials([o for _, o in parts])
+        got = [to_numpy(c, b["dtype"]) for c, b in zip(comb, spec["outputs"])]
+        assert_close_full(spec, ins, got, 0, kind="exact")
+
+
+@pytest.mark.parametrize("world", [2, 3, 8])
+def test_virtual_shard_cc_matmul_jacobi(world):
+    from paper_conf_sc_schulzegr25_b200 import to_numpy
+    spec = S.matmul(300, 200, 100)
+    x = G.matmul_inputs(300, 200, 100, "f32", "positive")
+    ref = oracle.evaluate(spec, x)[0]
+    for p, outs in _virtual_shards(spec, x, world, 0):
+        shp, off, _ = p.local_shape(True, 0)
+        g = to_numpy(outs[0], "f32").astype(np.float64)
+        r = ref[off[0]:off[0] + shp[0]]
+        assert (np.abs(g - r) / np.abs(r)).max() <= 1e-4
+    spec = S.jacobi3d(20, 12, 14)
+    x = G.jacobi3d_inputs(20, 12, 14)
+    ref = oracle.evaluate(spec, x)[0]
+    for p, outs in _virtual_shards(spec, x, world, 0):
+        shp, off, _ = p.local_shape(True, 0)
+        g = to_numpy(outs[0], "f32").astype(np.float64)
+        r = ref[off[0]:off[0] + shp[0]]
+        assert np.abs(g - r).max() <= 1e-4 * 2
