@@ -1,17 +1,436 @@
-// t4_tcgen05.cu — T4: bf16 tcgen05/TMEM contraction (placeholder until the kernel lands).
-#include "internal.h"
+// t4_tcgen05.cu — T4: bf16 contraction on the 5th-generation tensor cores (tcgen05/TMEM)
+// for f = MUL, ⊗ = pw(add) with reuse (MatMul Listing 9).
+//
+// Persistent, warp-specialised sm_100a kernel, one CTA per SM:
+//   warp 0       — TMA producer: cp.async.bulk.tensor 2-D loads of the A (128×64) and
+//                  B (64×256) bf16 tiles into a 4-stage 128-byte-swizzled smem ring,
+//                  completion counted on per-stage mbarriers (expect_tx);
+//   warp 1       — TMEM allocator + MMA issuer: one thread issues
+//                  tcgen05.mma.cta_group::1.kind::f16 (128×256×16, fp32 accumulate in
+//                  TMEM) on UMMA smem descriptors; tcgen05.commit frees smem stages and
+//                  signals the epilogue;
+//   warps 2..5   — epilogue: tcgen05.ld 32x32b.x32 TMEM → registers → global (fp32),
+//                  TMEM double-buffered (2 × 256 columns) so the epilogue of tile t
+//                  overlaps the MMAs of tile t+1.
+// Operands are described by 2-D tensor maps: an operand qualifies when its M (N) and K
+// offset tables are linear with one unit stride (K-major or MN-major; both are native
+// UMMA layouts for bf16).  M/N/K tails are TMA out-of-bounds zero fill + masked stores.
+// The output goes through the plan's offset tables (any affine out_view, e.g. the
+// 6-D CCSD(T) scatter) or, for a row-major C, as 16-byte vector stores.
+#include <cuda.h>
+#include <cudaTypedefs.h>
+
+#include <algorithm>
+#include <vector>
+
+#include "kcommon.cuh"
 
 namespace mdh {
 
-bool t4_supported(const Plan&, std::string* why) {
-  if (why) *why = "tcgen05 template not built yet";
-  return false;
+void build_contraction_tables(Plan* p, int64_t* a_kc, int64_t* b_kc);
+
+namespace t4 {
+
+constexpr int BM = 128, BN = 256, BK = 64, STAGES = 4;
+constexpr int THREADS = 192;
+constexpr int A_BYTES = BM * BK * 2;          // 16 KB
+constexpr int B_BYTES = BN * BK * 2;          // 32 KB
+constexpr int STAGE_BYTES = A_BYTES + B_BYTES;
+constexpr int SMEM_BYTES = STAGES * STAGE_BYTES + 1024 + 256;
+constexpr uint32_t TMEM_COLS = 512;           // 2 accumulators × 256 fp32 columns
+
+struct Params {
+  int64_t M, N, K;
+  int tiles_m, tiles_n, num_tiles, num_kb;
+  int a_mn_major, b_mn_major;
+  uint32_t idesc;
+  float* C;
+  int out_bf16;
+  int c_rowmajor;                   // C[m*ldc + n] fast path
+  int64_t ldc, cbase;
+  const int64_t* cM;                // generic output tables
+  const int64_t* cN;
+};
+
+__device__ __forceinline__ uint32_t smem_u32(const void* p) { return (uint32_t)__cvta_generic_to_shared(p); }
+
+__device__ __forceinline__ void mbar_init(uint32_t bar, uint32_t count) {
+  asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(bar), "r"(count));
 }
-mdh_status prepare_t4(Plan*) { set_error("T4 not available"); return MDH_ERR_UNSUPPORTED; }
-mdh_status launch_t4(const Plan&, const void* const*, void* const*, void*, cudaStream_t) {
-  set_error("T4 not available");
-  return MDH_ERR_UNSUPPORTED;
+__device__ __forceinline__ void mbar_wait(uint32_t bar, uint32_t parity) {
+  asm volatile(
+      "{\n\t.reg .pred p;\n\t"
+      "WAIT_%=:\n\t"
+      "mbarrier.try_wait.parity.shared::cta.b64 p, [%0], %1;\n\t"
+      "@!p bra WAIT_%=;\n\t}" ::"r"(bar),
+      "r"(parity)
+      : "memory");
 }
-void release_t4(Plan*) {}
+__device__ __forceinline__ void mbar_expect_tx(uint32_t bar, uint32_t bytes) {
+  asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(bar), "r"(bytes) : "memory");
+}
+__device__ __forceinline__ void mbar_arrive(uint32_t bar) {
+  asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(bar) : "memory");
+}
+__device__ __forceinline__ void tma_load_2d(uint32_t dst, const CUtensorMap* map, uint32_t bar, int c0, int c1) {
+  asm volatile(
+      "cp.async.bulk.tensor.2d.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1, {%3, %4}], [%2];" ::"r"(dst),
+      "l"((uint64_t)map), "r"(bar), "r"(c0), "r"(c1)
+      : "memory");
+}
+// UMMA shared-memory descriptor (sm_100): start>>4 [0,14), LBO>>4 [16,30), SBO>>4 [32,46),
+// version 1 [46,48), base offset 0, layout SWIZZLE_128B = 2 at [61,64).
+__device__ __forceinline__ uint64_t sdesc(uint32_t addr, uint32_t lbo, uint32_t sbo) {
+  return (uint64_t)((addr >> 4) & 0x3FFF) | ((uint64_t)((lbo >> 4) & 0x3FFF) << 16) |
+         ((uint64_t)((sbo >> 4) & 0x3FFF) << 32) | (1ull << 46) | (2ull << 61);
+}
+__device__ __forceinline__ void mma_bf16(uint32_t d_tmem, uint64_t a, uint64_t b, uint32_t idesc, uint32_t acc) {
+  asm volatile(
+      "{\n\t.reg .pred p;\n\tsetp.ne.b32 p, %4, 0;\n\t"
+      "tcgen05.mma.cta_group::1.kind::f16 [%0], %1, %2, %3, p;\n\t}" ::"r"(d_tmem),
+      "l"(a), "l"(b), "r"(idesc), "r"(acc));
+}
+__device__ __forceinline__ void mma_commit(uint32_t bar) {
+  asm volatile("tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.b64 [%0];" ::"r"(bar) : "memory");
+}
+__device__ __forceinline__ void tc_fence_before() { asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory"); }
+__device__ __forceinline__ void tc_fence_after() { asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory"); }
+
+__device__ __forceinline__ void tmem_ld32(uint32_t taddr, uint32_t* r) {
+  asm volatile(
+      "tcgen05.ld.sync.aligned.32x32b.x32.b32 "
+      "{%0,%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%15,"
+      "%16,%17,%18,%19,%20,%21,%22,%23,%24,%25,%26,%27,%28,%29,%30,%31}, [%32];"
+      : "=r"(r[0]), "=r"(r[1]), "=r"(r[2]), "=r"(r[3]), "=r"(r[4]), "=r"(r[5]), "=r"(r[6]), "=r"(r[7]), "=r"(r[8]),
+        "=r"(r[9]), "=r"(r[10]), "=r"(r[11]), "=r"(r[12]), "=r"(r[13]), "=r"(r[14]), "=r"(r[15]), "=r"(r[16]),
+        "=r"(r[17]), "=r"(r[18]), "=r"(r[19]), "=r"(r[20]), "=r"(r[21]), "=r"(r[22]), "=r"(r[23]), "=r"(r[24]),
+        "=r"(r[25]), "=r"(r[26]), "=r"(r[27]), "=r"(r[28]), "=r"(r[29]), "=r"(r[30]), "=r"(r[31])
+      : "r"(taddr));
+  asm volatile("tcgen05.wait::ld.sync.aligned;" ::: "memory");
+}
+
+__global__ void __launch_bounds__(THREADS, 1)
+    gemm_kernel(const __grid_constant__ CUtensorMap mapA, const __grid_constant__ CUtensorMap mapB,
+                const __grid_constant__ Params P) {
+  extern __shared__ __align__(1024) uint8_t smem_raw[];
+  uint8_t* smem = (uint8_t*)(((uintptr_t)smem_raw + 1023) & ~(uintptr_t)1023);
+  uint8_t* sA = smem;
+  uint8_t* sB = smem + STAGES * A_BYTES;
+  uint64_t* bars = (uint64_t*)(smem + STAGES * STAGE_BYTES);
+  // bars: full[STAGES], empty[STAGES], tmem_full[2], tmem_empty[2]; then the TMEM slot
+  uint32_t* tmem_slot = (uint32_t*)(bars + 2 * STAGES + 4);
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  const uint32_t full0 = smem_u32(bars), empty0 = smem_u32(bars + STAGES);
+  const uint32_t tfull0 = smem_u32(bars + 2 * STAGES), tempty0 = smem_u32(bars + 2 * STAGES + 2);
+
+  if (warp == 0 && lane == 0) {
+    asm volatile("prefetch.tensormap [%0];" ::"l"((uint64_t)&mapA) : "memory");
+    asm volatile("prefetch.tensormap [%0];" ::"l"((uint64_t)&mapB) : "memory");
+    for (int s = 0; s < STAGES; ++s) {
+      mbar_init(full0 + 8 * s, 1);
+      mbar_init(empty0 + 8 * s, 1);
+    }
+    for (int a = 0; a < 2; ++a) {
+      mbar_init(tfull0 + 8 * a, 1);
+      mbar_init(tempty0 + 8 * a, 128);
+    }
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+  }
+  if (warp == 1) {
+    asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(smem_u32(tmem_slot)),
+                 "r"(TMEM_COLS));
+    asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;");
+  }
+  tc_fence_before();
+  __syncthreads();
+  tc_fence_after();
+  const uint32_t tmem = *tmem_slot;
+
+  if (warp == 0) {
+    if (lane == 0) {
+      // ===== TMA producer =====
+      int stage = 0;
+      uint32_t phase = 0;
+      for (int t = blockIdx.x; t < P.num_tiles; t += gridDim.x) {
+        const int m0 = (t / P.tiles_n) * BM, n0 = (t % P.tiles_n) * BN;
+        for (int kb = 0; kb < P.num_kb; ++kb) {
+          mbar_wait(empty0 + 8 * stage, phase ^ 1);
+          const uint32_t fb = full0 + 8 * stage;
+          mbar_expect_tx(fb, STAGE_BYTES);
+          const uint32_t a_dst = smem_u32(sA + stage * A_BYTES), b_dst = smem_u32(sB + stage * B_BYTES);
+          const int k0 = kb * BK;
+          if (P.a_mn_major) {          // box {64 m, 64 k}, two atoms along M
+            tma_load_2d(a_dst, &mapA, fb, m0, k0);
+            tma_load_2d(a_dst + 8192, &mapA, fb, m0 + 64, k0);
+          } else {                     // box {64 k, 128 m}
+            tma_load_2d(a_dst, &mapA, fb, k0, m0);
+          }
+          if (P.b_mn_major) {          // box {64 n, 64 k}, four atoms along N
+#pragma unroll
+            for (int j = 0; j < 4; ++j) tma_load_2d(b_dst + 8192 * j, &mapB, fb, n0 + 64 * j, k0);
+          } else {                     // box {64 k, 256 n}
+            tma_load_2d(b_dst, &mapB, fb, k0, n0);
+          }
+          if (++stage == STAGES) { stage = 0; phase ^= 1; }
+        }
+      }
+    }
+  } else if (warp == 1) {
+    if (lane == 0) {
+      // ===== MMA issuer (one thread) =====
+      int stage = 0;
+      uint32_t phase = 0;
+      int it = 0;
+      for (int t = blockIdx.x; t < P.num_tiles; t += gridDim.x, ++it) {
+        const int acc = it & 1;
+        mbar_wait(tempty0 + 8 * acc, ((it >> 1) & 1) ^ 1);
+        tc_fence_after();
+        const uint32_t d = tmem + acc * BN;
+        for (int kb = 0; kb < P.num_kb; ++kb) {
+          mbar_wait(full0 + 8 * stage, phase);
+          tc_fence_after();
+          const uint32_t a0 = smem_u32(sA + stage * A_BYTES), b0 = smem_u32(sB + stage * B_BYTES);
+#pragma unroll
+          for (int k = 0; k < BK / 16; ++k) {
+            // K-major: +32 B per 16-element K step inside the 128-B swizzled row;
+            // MN-major: +16 rows × 128 B = 2048 B per K step (LBO = next 64-wide MN atom)
+            const uint64_t ad = P.a_mn_major ? sdesc(a0 + 2048 * k, 8192, 1024) : sdesc(a0 + 32 * k, 16, 1024);
+            const uint64_t bd = P.b_mn_major ? sdesc(b0 + 2048 * k, 8192, 1024) : sdesc(b0 + 32 * k, 16, 1024);
+            mma_bf16(d, ad, bd, P.idesc, (kb | k) != 0);
+          }
+          mma_commit(empty0 + 8 * stage);            // smem stage free once these MMAs retire
+          if (++stage == STAGES) { stage = 0; phase ^= 1; }
+        }
+        mma_commit(tfull0 + 8 * acc);                 // accumulator ready for the epilogue
+      }
+    }
+  } else {
+    // ===== epilogue: warps 2..5 → TMEM lane quadrant (warp % 4) =====
+    const int quad = warp & 3;
+    const int row = quad * 32 + lane;
+    int it = 0;
+    for (int t = blockIdx.x; t < P.num_tiles; t += gridDim.x, ++it) {
+      const int acc = it & 1;
+      const int64_t m = (int64_t)(t / P.tiles_n) * BM + row;
+      const int64_t n0 = (int64_t)(t % P.tiles_n) * BN;
+      mbar_wait(tfull0 + 8 * acc, (it >> 1) & 1);
+      tc_fence_after();
+      const bool mok = m < P.M;
+      const int64_t crow = mok ? (P.c_rowmajor ? P.cbase + m * P.ldc : P.cbase + P.cM[m]) : 0;
+#pragma unroll 1
+      for (int c = 0; c < BN / 32; ++c) {
+        uint32_t r[32];
+        tmem_ld32(tmem + ((uint32_t)(quad * 32) << 16) + acc * BN + c * 32, r);
+        if (!mok) continue;
+        const int64_t nb = n0 + c * 32;
+        if (P.c_rowmajor && !P.out_bf16 && nb + 32 <= P.N && ((crow + nb) & 3) == 0) {
+          float4* dst = reinterpret_cast<float4*>(P.C + crow + nb);
+#pragma unroll
+          for (int j = 0; j < 8; ++j)
+            dst[j] = make_float4(__uint_as_float(r[4 * j]), __uint_as_float(r[4 * j + 1]), __uint_as_float(r[4 * j + 2]),
+                                 __uint_as_float(r[4 * j + 3]));
+        } else {
+#pragma unroll
+          for (int j = 0; j < 32; ++j) {
+            const int64_t n = nb + j;
+            if (n < P.N) {
+              const int64_t o = crow + (P.c_rowmajor ? n : P.cN[n]);
+              if (P.out_bf16) ((__nv_bfloat16*)P.C)[o] = __float2bfloat16_rn(__uint_as_float(r[j]));
+              else P.C[o] = __uint_as_float(r[j]);
+            }
+          }
+        }
+      }
+      tc_fence_before();
+      mbar_arrive(tempty0 + 8 * acc);
+    }
+  }
+  tc_fence_before();
+  __syncthreads();
+  if (warp == 1) {
+    tc_fence_after();
+    asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" ::"r"(tmem), "r"(TMEM_COLS));
+  }
+}
+
+// ------------------------------------------------------------------------- host
+struct Layout2D {
+  bool ok = false;
+  bool mn_major = false;       // unit stride along M (N) instead of K
+  int64_t ld = 0;              // stride (elements) of the non-unit dim
+};
+
+static bool linear(const std::vector<int64_t>& t, int64_t* stride) {
+  if (t.size() <= 1) { *stride = 0; return true; }
+  int64_t s = t[1] - t[0];
+  for (size_t i = 1; i < t.size(); ++i)
+    if (t[i] - t[i - 1] != s) return false;
+  *stride = s;
+  return true;
+}
+
+static std::vector<int64_t> table(const Plan& p, const int* dims, int nd, const Access& acc) {
+  int64_t n = 1;
+  for (int t = 0; t < nd; ++t) n *= p.size[dims[t]];
+  std::vector<int64_t> tab((size_t)n);
+  for (int64_t q = 0; q < n; ++q) {
+    int64_t rem = q, off = 0;
+    for (int t = nd - 1; t >= 0; --t) {
+      int64_t v = rem % p.size[dims[t]];
+      rem /= p.size[dims[t]];
+      off += acc.L[dims[t]] * v;
+    }
+    tab[(size_t)q] = off;
+  }
+  return tab;
+}
+
+static Layout2D operand_layout(const Plan& p, const int* mdims, int nmd, int64_t MN, const Access& acc, std::string* why,
+                               const char* name) {
+  Layout2D L;
+  int64_t smn, sk;
+  const Contraction& c = p.con;
+  if (!linear(table(p, mdims, nmd, acc), &smn) || !linear(table(p, c.kd, c.nk, acc), &sk)) {
+    *why = std::string(name) + " offsets are not 2-D linear";
+    return L;
+  }
+  if (MN == 1) smn = 1;
+  if (c.K == 1) sk = 1;
+  if (sk == 1 && (smn * 2) % 16 == 0 && smn > 0) { L.ok = true; L.mn_major = false; L.ld = smn; }
+  else if (smn == 1 && (sk * 2) % 16 == 0 && sk > 0) { L.ok = true; L.mn_major = true; L.ld = sk; }
+  else *why = std::string(name) + " has no unit stride with a 16-byte aligned leading dimension (TMA)";
+  return L;
+}
+
+}  // namespace t4
+
+bool t4_supported(const Plan& p, std::string* why) {
+  const Contraction& c = p.con;
+  if (c.Z != 1) { *why = "batched contraction (Z>1) not in the tcgen05 template yet"; return false; }
+  if (p.out[0].dtype != MDH_F32 && p.out[0].dtype != MDH_BF16) { *why = "output must be f32/bf16"; return false; }
+  if (p.in[c.a_buf].acc[0].base % 8 || p.in[c.b_buf].acc[0].base % 8) { *why = "operand base not 16-byte aligned"; return false; }
+  t4::Layout2D a = t4::operand_layout(p, c.md, c.nm, c.M, p.in[c.a_buf].acc[0], why, "A");
+  if (!a.ok) return false;
+  t4::Layout2D b = t4::operand_layout(p, c.nd, c.nn, c.N, p.in[c.b_buf].acc[0], why, "B");
+  if (!b.ok) return false;
+  if (c.M > INT32_MAX || c.N > INT32_MAX || c.K > INT32_MAX) { *why = "extent exceeds TMA coordinates"; return false; }
+  *why = std::string("A ") + (a.mn_major ? "MN" : "K") + "-major, B " + (b.mn_major ? "MN" : "K") + "-major";
+  return true;
+}
+
+struct T4State {
+  t4::Layout2D a, b;
+  t4::Params P;
+};
+
+mdh_status prepare_t4(Plan* p) {
+  std::string why;
+  if (!t4_supported(*p, &why)) { set_error("T4: %s", why.c_str()); return MDH_ERR_UNSUPPORTED; }
+  const Contraction& c = p->con;
+  T4State* s = new T4State();
+  s->a = t4::operand_layout(*p, c.md, c.nm, c.M, p->in[c.a_buf].acc[0], &why, "A");
+  s->b = t4::operand_layout(*p, c.nd, c.nn, c.N, p->in[c.b_buf].acc[0], &why, "B");
+  int64_t akc, bkc;
+  p->host_const.clear();
+  build_contraction_tables(p, &akc, &bkc);
+  t4::Params& P = s->P;
+  memset(&P, 0, sizeof(P));
+  P.M = c.M;
+  P.N = c.N;
+  P.K = c.K;
+  P.tiles_m = (int)((c.M + t4::BM - 1) / t4::BM);
+  P.tiles_n = (int)((c.N + t4::BN - 1) / t4::BN);
+  P.num_tiles = P.tiles_m * P.tiles_n;
+  P.num_kb = (int)((c.K + t4::BK - 1) / t4::BK);
+  P.a_mn_major = s->a.mn_major;
+  P.b_mn_major = s->b.mn_major;
+  // instruction descriptor (kind::f16): D f32, A/B bf16, majors, N>>3, M>>4
+  P.idesc = (1u << 4) | (1u << 7) | (1u << 10) | ((uint32_t)P.a_mn_major << 15) | ((uint32_t)P.b_mn_major << 16) |
+            ((uint32_t)(t4::BN >> 3) << 17) | ((uint32_t)(t4::BM >> 4) << 24);
+  P.out_bf16 = p->out[0].dtype == MDH_BF16;
+  // is C row-major over (m, n)?  cM[m] = m*ldc, cN[n] = n
+  std::vector<int64_t> cm = t4::table(*p, c.md, c.nm, p->out[0].acc[0]);
+  std::vector<int64_t> cn = t4::table(*p, c.nd, c.nn, p->out[0].acc[0]);
+  int64_t sm = 0, sn = 0;
+  bool lm = t4::linear(cm, &sm), ln = t4::linear(cn, &sn);
+  if (c.N == 1) sn = 1;
+  P.c_rowmajor = lm && ln && sn == 1 && cm[0] == 0 && cn[0] == 0;
+  P.ldc = sm;
+  P.cbase = p->out[0].acc[0].base;
+  p->tmaps = s;
+  p->t4_variant = 1;
+  p->ws_kernel = 0;
+  p->tiles.bm = t4::BM;
+  p->tiles.bn = t4::BN;
+  p->tiles.bk = t4::BK;
+  p->tiles.stages = t4::STAGES;
+  return MDH_OK;
+}
+
+void release_t4(Plan* p) {
+  if (p->tmaps) {
+    delete (T4State*)p->tmaps;
+    p->tmaps = nullptr;
+  }
+}
+
+static PFN_cuTensorMapEncodeTiled_v12000 encode_fn() {
+  static PFN_cuTensorMapEncodeTiled_v12000 fn = nullptr;
+  static std::once_flag once;
+  std::call_once(once, [] {
+    void* f = nullptr;
+    cudaDriverEntryPointQueryResult q;
+    if (cudaGetDriverEntryPoint("cuTensorMapEncodeTiled", &f, cudaEnableDefault, &q) == cudaSuccess &&
+        q == cudaDriverEntryPointSuccess)
+      fn = (PFN_cuTensorMapEncodeTiled_v12000)f;
+  });
+  return fn;
+}
+
+// 2-D bf16 tensor map: inner dim `inner` (unit stride), outer dim `outer` with stride ld
+static mdh_status make_map(CUtensorMap* map, const void* base, int64_t inner, int64_t outer, int64_t ld, uint32_t box_in,
+                           uint32_t box_out) {
+  auto fn = encode_fn();
+  if (!fn) { set_error("cuTensorMapEncodeTiled unavailable (driver too old?)"); return MDH_ERR_CUDA; }
+  cuuint64_t dims[2] = {(cuuint64_t)inner, (cuuint64_t)std::max<int64_t>(outer, 1)};
+  cuuint64_t strides[1] = {(cuuint64_t)(std::max<int64_t>(ld, inner) * 2)};
+  cuuint32_t box[2] = {box_in, box_out};
+  cuuint32_t estr[2] = {1, 1};
+  CUresult r = fn(map, CU_TENSOR_MAP_DATA_TYPE_BFLOAT16, 2, const_cast<void*>(base), dims, strides, box, estr,
+                  CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_128B, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
+                  CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+  if (r != CUDA_SUCCESS) { set_error("cuTensorMapEncodeTiled failed (%d)", (int)r); return MDH_ERR_CUDA; }
+  return MDH_OK;
+}
+
+mdh_status launch_t4(const Plan& p, const void* const* in, void* const* out, void*, cudaStream_t st) {
+  const char* dc = nullptr;
+  MDH_TRY(device_consts(p, &dc));
+  const T4State* s = (const T4State*)p.tmaps;
+  const Contraction& c = p.con;
+  t4::Params P = s->P;
+  P.C = (float*)out[0];
+  P.cM = (const int64_t*)(dc + p.tab_off[4]);
+  P.cN = (const int64_t*)(dc + p.tab_off[5]);
+  const uint16_t* A = (const uint16_t*)in[c.a_buf] + p.in[c.a_buf].acc[0].base;
+  const uint16_t* B = (const uint16_t*)in[c.b_buf] + p.in[c.b_buf].acc[0].base;
+  CUtensorMap ma, mb;
+  if (s->a.mn_major) MDH_TRY(make_map(&ma, A, c.M, c.K, s->a.ld, 64, 64));
+  else MDH_TRY(make_map(&ma, A, c.K, c.M, s->a.ld, 64, 128));
+  if (s->b.mn_major) MDH_TRY(make_map(&mb, B, c.N, c.K, s->b.ld, 64, 64));
+  else MDH_TRY(make_map(&mb, B, c.K, c.N, s->b.ld, 64, 256));
+  static std::once_flag attr_once;
+  static cudaError_t attr_err = cudaSuccess;
+  std::call_once(attr_once, [] {
+    attr_err = cudaFuncSetAttribute(t4::gemm_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, t4::SMEM_BYTES);
+  });
+  MDH_CUDA(attr_err);
+  int dev = 0, sms = 148;
+  cudaGetDevice(&dev);
+  cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+  const int grid = std::min(P.num_tiles, sms);
+  t4::gemm_kernel<<<grid, t4::THREADS, t4::SMEM_BYTES, st>>>(ma, mb, P);
+  return post_launch("t4_gemm_kernel");
+}
 
 }  // namespace mdh

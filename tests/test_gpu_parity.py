@@ -132,7 +132,8 @@ def test_matmul_fp32(mnk):
     spec = S.matmul(M, N, K)
     x = G.matmul_inputs(M, N, K, "f32", "positive")
     got, p = run_gpu(spec, x)
-    assert p.template == "T3_simt_contraction"
+    # degenerate 1-point dims carry no M/N group, so (1,1,1) is a plain reduction
+    assert p.template == ("T2_reduce" if M == 1 or N == 1 else "T3_simt_contraction")
     assert_close_full(spec, x, got, 1e-4, kind="rel")
 
 
@@ -327,3 +328,42 @@ def test_virtual_shard_cc_matmul_jacobi(world):
         g = to_numpy(outs[0], "f32").astype(np.float64)
         r = ref[off[0]:off[0] + shp[0]]
         assert np.abs(g - r).max() <= 1e-4 * 2
+
+
+# ----------------------------------------------------------------- T4: tcgen05 contraction
+def _mm_spec(M, N, K, a_t=False, b_t=False, out="f32"):
+    d = ["i", "j", "k"]
+    a = ["k", "i"] if a_t else ["i", "k"]
+    b = ["j", "k"] if b_t else ["k", "j"]
+    return S.make_spec("mm", d, [M, N, K], ["CC", "CC", "PW_ADD"], "MUL",
+                       [S.buffer("A", "bf16", [a], d), S.buffer("B", "bf16", [b], d)],
+                       [S.buffer("C", out, [["i", "j"]], d)])
+
+
+@pytest.mark.parametrize("mnk", [(128, 256, 64), (256, 512, 128), (300, 200, 1000), (8, 8, 8), (1000, 1032, 72)])
+@pytest.mark.parametrize("at,bt", [(False, False), (False, True), (True, False), (True, True)])
+def test_matmul_bf16_tcgen05(mnk, at, bt):
+    M, N, K = mnk
+    spec = _mm_spec(M, N, K, at, bt)
+    x = G.gen_inputs(spec, 3100, "positive")
+    got, p = run_gpu(spec, x)
+    # TMA needs a 16-byte aligned leading dimension: A^T needs M%8==0, A needs K%8==0, etc.
+    lda = M if at else K
+    ldb = K if bt else N
+    tma_ok = lda % 8 == 0 and ldb % 8 == 0
+    assert p.template == ("T4_tcgen05_contraction" if tma_ok else "T3_simt_contraction"), p.describe()
+    assert_close_full(spec, x, got, 1e-2, kind="rel")
+
+
+def test_matmul_bf16_full_size():
+    spec = S.matmul(4096, 4096, 4096, "bf16")
+    x = G.matmul_inputs(4096, 4096, 4096, "bf16", "signed")
+    got, p = run_gpu(spec, x)
+    assert p.template == "T4_tcgen05_contraction"
+    assert_close_points(spec, x, got, 1e-2, n=3000, kind="scale")
+    x = G.matmul_inputs(4096, 4096, 4096, "bf16", "ones")
+    got, _ = run_gpu(spec, x)
+    assert np.all(got[0] == 4096.0)
+    x = G.matmul_inputs(4096, 4096, 4096, "bf16", "identity")
+    got, _ = run_gpu(spec, x)
+    assert np.array_equal(got[0], G.bf16_bits_to_f32(x[1]))
