@@ -148,7 +148,11 @@ typedef struct mdh_plan_s* mdh_plan_t;
  * Errors: INVALID_SPEC / UNSUPPORTED as described above; INVALID_ARG for bad opts. */
 mdh_status mdh_plan(const mdh_spec* spec, const mdh_plan_opts* opts, mdh_plan_t* plan_out);
 
-/* Device workspace the caller must pass to mdh_execute (bytes, 256-B aligned start). */
+/* Device workspace the caller must pass to mdh_execute (bytes, 256-B aligned start).
+ * The workspace must be ZERO-FILLED before its first use with a plan (e.g. one
+ * cudaMemsetAsync); every mdh_execute leaves it zero-filled again where it matters
+ * (the cross-CTA combine tickets reset themselves), so it can be reused without
+ * re-initialisation.  One workspace must not be used by two concurrent executes. */
 mdh_status mdh_plan_workspace_size(mdh_plan_t plan, size_t* bytes);
 
 /* The shape of input (is_output=0) or output (is_output=1) buffer `buf` as THIS rank

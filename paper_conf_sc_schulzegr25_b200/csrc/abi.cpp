@@ -271,6 +271,7 @@ mdh_status mdh_execute_host(mdh_plan_t plan, const void* const* host_in, void* c
     off += (n + 255) / 256 * 256;
   }
   void* ws = base + off;
+  if (p.ws_total) MDH_CUDA(cudaMemsetAsync(ws, 0, p.ws_total, st));   // workspace contract
   mdh_status s = mdh_execute(plan, din, dout, ws, p.ws_total, cuda_stream);
   if (s != MDH_OK) return s;
   int launched = mdh::launch_count();

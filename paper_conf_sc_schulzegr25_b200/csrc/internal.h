@@ -108,6 +108,8 @@ struct Plan {
   mutable std::mutex mu;
   void* tmaps = nullptr;              // T4: host copy of CUtensorMap descriptors
   int t4_variant = 0;
+  std::vector<int64_t> auxi;          // template-specific host data (e.g. T1 stencil shape)
+  std::vector<double> auxd;
 };
 
 // device pointer of the plan's constants (uploads them on first use)

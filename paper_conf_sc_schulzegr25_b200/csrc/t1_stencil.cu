@@ -66,7 +66,124 @@ __global__ void __launch_bounds__(256) t1_kernel(const __grid_constant__ T1Param
   }
 }
 
+// ---- specialised 7-point cross (radius 1, "j3d7pt", reading C-16) ----------------------
+// Each thread owns 4 consecutive x outputs of one y row and marches z.  The centre row
+// segment (x0-1 … x0+4) of planes z-1, z, z+1 lives in a register queue, so a z step
+// loads only the new centre row of plane z+1 plus the y-1 / y+1 rows of plane z — six
+// 128/64-bit loads per 4 outputs (instead of 28 scalar loads); x±1 come from the centre
+// row registers.  Every input element is read from HBM once (the y±1 re-reads of
+// neighbouring threads hit L1/L2).
+struct J7Params {
+  const float* u;
+  float* v;
+  int64_t bc;              // element offset of the centre access at the origin
+  int64_t Ly, Lz;          // input strides of y and z (x stride 1)
+  int64_t ob, oLy, oLz;    // output (x stride 1)
+  int X, Y, Z, zchunk;
+  float wc, wxm, wxp, wym, wyp, wzm, wzp;
+};
+
+template <bool VEC>
+__device__ __forceinline__ void row6(const float* p, bool full, int64_t rem, float r[6]) {
+  // r[k] = p[k], k = 0..5  (p = the x0-1 position); rem = number of valid positions
+  if (VEC && full) {
+    const float4 a = __ldg(reinterpret_cast<const float4*>(p));
+    const float2 b = __ldg(reinterpret_cast<const float2*>(p + 4));
+    r[0] = a.x; r[1] = a.y; r[2] = a.z; r[3] = a.w; r[4] = b.x; r[5] = b.y;
+  } else {
+#pragma unroll
+    for (int k = 0; k < 6; ++k) r[k] = k < rem ? __ldg(p + k) : 0.f;
+  }
+}
+
+template <bool VEC_IN, bool VEC_OUT>
+__global__ void __launch_bounds__(128) t1_j3d7_kernel(const __grid_constant__ J7Params P) {
+  const int x0 = (blockIdx.x * 32 + threadIdx.x) * 4;
+  const int y = blockIdx.y * 4 + threadIdx.y;
+  if (x0 >= P.X || y >= P.Y) return;
+  const int z0 = blockIdx.z * P.zchunk;
+  const int z1 = min(P.Z, z0 + P.zchunk);
+  const bool full = x0 + 4 <= P.X;
+  const int64_t rem = (int64_t)P.X + 1 - x0 + 1;     // valid positions x0-1 … X (centre-relative)
+  const float* pc = P.u + P.bc - 1 + x0 + (int64_t)y * P.Ly + (int64_t)z0 * P.Lz;
+  float* po = P.v + P.ob + x0 + (int64_t)y * P.oLy + (int64_t)z0 * P.oLz;
+  float rm[6], r0[6], rp[6], ym[6], yp[6];
+  row6<VEC_IN>(pc - P.Lz, full, rem, rm);
+  row6<VEC_IN>(pc, full, rem, r0);
+  for (int z = z0; z < z1; ++z) {
+    row6<VEC_IN>(pc + P.Lz, full, rem, rp);
+    row6<VEC_IN>(pc - P.Ly, full, rem, ym);
+    row6<VEC_IN>(pc + P.Ly, full, rem, yp);
+    float o[4];
+#pragma unroll
+    for (int j = 0; j < 4; ++j) {
+      float acc = P.wc * r0[j + 1];
+      acc = fmaf(P.wxm, r0[j], acc);
+      acc = fmaf(P.wxp, r0[j + 2], acc);
+      acc = fmaf(P.wym, ym[j + 1], acc);
+      acc = fmaf(P.wyp, yp[j + 1], acc);
+      acc = fmaf(P.wzm, rm[j + 1], acc);
+      acc = fmaf(P.wzp, rp[j + 1], acc);
+      o[j] = acc;
+    }
+    if (VEC_OUT && full) {
+      reinterpret_cast<float2*>(po)[0] = make_float2(o[0], o[1]);
+      reinterpret_cast<float2*>(po)[1] = make_float2(o[2], o[3]);
+    } else {
+#pragma unroll
+      for (int j = 0; j < 4; ++j)
+        if (x0 + j < P.X) po[j] = o[j];
+    }
+#pragma unroll
+    for (int k = 0; k < 6; ++k) { rm[k] = r0[k]; r0[k] = rp[k]; }
+    pc += P.Lz;
+    po += P.oLz;
+  }
+}
+
+// Recognise the 7-point cross: one fp32 input buffer, 7 accesses sharing the linear part
+// (x stride 1), shifts = centre ± one unit in exactly one of x, y, z.  Stores in auxi:
+// [dz_dim, dy_dim, dx_dim, centre access, index of access for xm,xp,ym,yp,zm,zp].
+static bool detect_j3d7(Plan* p) {
+  if (p->n_in != 1 || p->in[0].nacc != 7 || p->in[0].dtype != MDH_F32 || p->f != MDH_F_STENCIL) return false;
+  if (p->out[0].dtype != MDH_F32) return false;
+  int dims[3], nd = 0;
+  for (int d = 0; d < p->D; ++d)
+    if (p->size[d] > 1) { if (nd == 3) return false; dims[nd++] = d; }
+  if (nd != 3) return false;
+  const int dz = dims[0], dy = dims[1], dx = dims[2];
+  const Buf& B = p->in[0];
+  for (int a = 1; a < 7; ++a)
+    for (int d = 0; d < p->D; ++d)
+      if (B.acc[a].L[d] != B.acc[0].L[d]) return false;
+  const int64_t Lx = B.acc[0].L[dx], Ly = B.acc[0].L[dy], Lz = B.acc[0].L[dz];
+  if (Lx != 1 || Ly < 4 || Lz < 3 * Ly) return false;
+  const Access& O = p->out[0].acc[0];
+  if (O.L[dx] != 1) return false;
+  for (int c = 0; c < 7; ++c) {
+    int idx[6] = {-1, -1, -1, -1, -1, -1};
+    bool ok = true;
+    for (int a = 0; a < 7 && ok; ++a) {
+      if (a == c) continue;
+      int64_t s = B.acc[a].base - B.acc[c].base;
+      int k = s == -1 ? 0 : s == 1 ? 1 : s == -Ly ? 2 : s == Ly ? 3 : s == -Lz ? 4 : s == Lz ? 5 : -1;
+      if (k < 0 || idx[k] >= 0) ok = false; else idx[k] = a;
+    }
+    if (!ok) continue;
+    p->auxi = {dz, dy, dx, c, idx[0], idx[1], idx[2], idx[3], idx[4], idx[5]};
+    return true;
+  }
+  return false;
+}
+
 mdh_status prepare_t1(Plan* p) {
+  p->auxi.clear();
+  if (detect_j3d7(p)) {
+    p->ws_kernel = 0;
+    p->t4_variant = 0;
+    p->why += " [7-point cross register-queue kernel]";
+    return MDH_OK;
+  }
   // fast path: fp32 inputs, <= 3 non-degenerate dims, <= 32 accesses; else generic
   bool ok = p->compute == MDH_F32 && p->n_in_acc <= T1_MAX_ACC && p->n_out == 1 && p->out[0].nacc == 1;
   for (int b = 0; b < p->n_in; ++b) ok &= p->in[b].dtype == MDH_F32;
@@ -82,7 +199,42 @@ mdh_status prepare_t1(Plan* p) {
   return MDH_OK;
 }
 
+static mdh_status launch_j3d7(const Plan& p, const void* const* in, void* const* out, cudaStream_t st) {
+  J7Params P;
+  memset(&P, 0, sizeof(P));
+  const int dz = (int)p.auxi[0], dy = (int)p.auxi[1], dx = (int)p.auxi[2], c = (int)p.auxi[3];
+  const Buf& B = p.in[0];
+  const Access& O = p.out[0].acc[0];
+  P.u = (const float*)in[0];
+  P.v = (float*)out[0];
+  P.bc = B.acc[c].base;
+  P.Ly = B.acc[c].L[dy];
+  P.Lz = B.acc[c].L[dz];
+  P.ob = O.base;
+  P.oLy = O.L[dy];
+  P.oLz = O.L[dz];
+  P.X = (int)p.size[dx];
+  P.Y = (int)p.size[dy];
+  P.Z = (int)p.size[dz];
+  P.wc = (float)p.fparams[c];
+  float* w[6] = {&P.wxm, &P.wxp, &P.wym, &P.wyp, &P.wzm, &P.wzp};
+  for (int k = 0; k < 6; ++k) *w[k] = (float)p.fparams[p.auxi[4 + k]];
+  int zc = p.tiles.zchunk > 0 ? p.tiles.zchunk : 64;
+  if (zc > P.Z) zc = P.Z;
+  P.zchunk = zc;
+  const bool vin = (P.bc - 1) % 4 == 0 && P.Ly % 4 == 0 && P.Lz % 4 == 0;
+  const bool vout = P.ob % 2 == 0 && P.oLy % 2 == 0 && P.oLz % 2 == 0;
+  dim3 block(32, 4);
+  dim3 grid((unsigned)((P.X + 127) / 128), (unsigned)((P.Y + 3) / 4), (unsigned)((P.Z + zc - 1) / zc));
+  if (vin && vout) t1_j3d7_kernel<true, true><<<grid, block, 0, st>>>(P);
+  else if (vin) t1_j3d7_kernel<true, false><<<grid, block, 0, st>>>(P);
+  else if (vout) t1_j3d7_kernel<false, true><<<grid, block, 0, st>>>(P);
+  else t1_j3d7_kernel<false, false><<<grid, block, 0, st>>>(P);
+  return post_launch("t1_j3d7_kernel");
+}
+
 mdh_status launch_t1(const Plan& p, const void* const* in, void* const* out, void*, cudaStream_t st) {
+  if (!p.auxi.empty()) return launch_j3d7(p, in, out, st);
   T1Params P;
   memset(&P, 0, sizeof(P));
   // map the (up to 3) non-degenerate dims to z, y, x in dimension order (x = last)

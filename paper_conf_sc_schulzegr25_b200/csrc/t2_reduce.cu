@@ -189,6 +189,69 @@ __global__ void __launch_bounds__(256) t2_row_kernel(const __grid_constant__ T2P
   }
 }
 
+// warp mode (S == 1, moderate contiguous rows, many cc points: MatVec): one warp per
+// cc point, 128-bit loads with 4 vectors in flight per lane, shuffle tree, no smem.
+template <class TI, class V, int OP, int F>
+__global__ void __launch_bounds__(256) t2_warp_kernel(const __grid_constant__ T2Params P) {
+  const TI* A = (const TI*)P.a;
+  const TI* B = (const TI*)P.b;
+  constexpr int W = VecOf<TI>::W;
+  const int lane = threadIdx.x & 31;
+  const int64_t warps = (int64_t)gridDim.x * (blockDim.x >> 5);
+  for (int64_t c = blockIdx.x * (int64_t)(blockDim.x >> 5) + (threadIdx.x >> 5); c < P.Ncc; c += warps) {
+    int64_t ao = P.abase, bo = P.bbase, oo = P.obase, rem = c;
+    for (int t = P.ncc - 1; t >= 0; --t) {
+      int64_t v = rem % P.ccsize[t];
+      rem /= P.ccsize[t];
+      ao += P.aLc[t] * v;
+      bo += P.bLc[t] * v;
+      oo += P.oLc[t] * v;
+    }
+    V acc0 = identity_t<OP, V>(), acc1 = acc0, acc2 = acc0, acc3 = acc0;
+    int64_t r = 0;
+    const int64_t r1 = P.Nred;
+    if (F != MDH_F_MUL || ((ao - bo) % W) == 0) {
+      int64_t mis = ((ao % W) + W) % W;
+      int64_t head = mis ? min((int64_t)(W - mis), r1) : (int64_t)0;
+      if (lane < head) {
+        V y = (F == MDH_F_MUL) ? Arith<V>::mul(cvt<TI, V>(ld1(A + ao + lane)), cvt<TI, V>(ld1(B + bo + lane)))
+                               : cvt<TI, V>(ld1(A + ao + lane));
+        acc0 = combine_t<OP, V>(acc0, y);
+      }
+      r = head;
+      const int64_t nvec = (r1 - r) / W;
+      const uint4* va = reinterpret_cast<const uint4*>(A + ao + r);
+      const uint4* vb = reinterpret_cast<const uint4*>(B + bo + r);
+      int64_t v = lane;
+      for (; v + 96 < nvec; v += 128) {
+        uint4 a0 = ld_nc_v4(va + v), a1 = ld_nc_v4(va + v + 32), a2 = ld_nc_v4(va + v + 64), a3 = ld_nc_v4(va + v + 96);
+        uint4 b0 = a0, b1 = a1, b2 = a2, b3 = a3;
+        if (F == MDH_F_MUL) {
+          b0 = __ldg(vb + v); b1 = __ldg(vb + v + 32); b2 = __ldg(vb + v + 64); b3 = __ldg(vb + v + 96);
+        }
+        acc0 = fold_vec<TI, V, OP, F>(acc0, a0, b0);
+        acc1 = fold_vec<TI, V, OP, F>(acc1, a1, b1);
+        acc2 = fold_vec<TI, V, OP, F>(acc2, a2, b2);
+        acc3 = fold_vec<TI, V, OP, F>(acc3, a3, b3);
+      }
+      for (; v < nvec; v += 32) {
+        uint4 a0 = ld_nc_v4(va + v);
+        uint4 b0 = (F == MDH_F_MUL) ? __ldg(vb + v) : a0;
+        acc0 = fold_vec<TI, V, OP, F>(acc0, a0, b0);
+      }
+      r += nvec * W;
+    }
+    for (int64_t k = r + lane; k < r1; k += 32) {
+      V y = (F == MDH_F_MUL) ? Arith<V>::mul(cvt<TI, V>(ld1(A + ao + k)), cvt<TI, V>(ld1(B + bo + k)))
+                             : cvt<TI, V>(ld1(A + ao + k));
+      acc1 = combine_t<OP, V>(acc1, y);
+    }
+    V acc = combine_t<OP, V>(combine_t<OP, V>(acc0, acc1), combine_t<OP, V>(acc2, acc3));
+    acc = warp_reduce<OP, V>(acc);
+    if (lane == 0) store_as<V>(P.out, P.odt, oo, acc);
+  }
+}
+
 template <class TI, class V, int OP, int F>
 __global__ void __launch_bounds__(256) t2_col_kernel(const __grid_constant__ T2Params P) {
   const TI* A = (const TI*)P.a;
@@ -278,7 +341,8 @@ mdh_status prepare_t2(Plan* p) {
   if (p->tiles.split > 0) S = (int)std::min<int64_t>(p->tiles.split, p->Nred);
   if (S < 1) S = 1;
   p->tiles.split = S;
-  p->tiles.vec = row ? 1 : 0;    // 1 = row mode
+  // 0 = column mode, 1 = row mode (CTA per unit), 2 = row mode (warp per cc point)
+  p->tiles.vec = row ? ((S == 1 && p->Nred <= 65536 && p->Ncc >= 148 * 8) ? 2 : 1) : 0;
   size_t part = (S > 1) ? (size_t)p->Ncc * S * compute_size(*p) : 0;
   size_t tick = (S > 1 && row) ? (size_t)p->Ncc * 4 : 0;
   p->ws_kernel = (part + 255) / 256 * 256 + (tick + 255) / 256 * 256;
@@ -290,6 +354,21 @@ static mdh_status launch_typed(const Plan& p, const T2Params& P, cudaStream_t st
   const bool row = p.tiles.vec == 1;
   const int F = p.f;
   int64_t units = P.Ncc * P.S;
+  if (p.tiles.vec == 2) {
+    unsigned g = (unsigned)std::min<int64_t>((P.Ncc + 7) / 8, 148LL * 16);
+#define T2_WARP(OP, FF) t2_warp_kernel<TI, V, OP, FF><<<g, 256, 0, st>>>(P)
+    if (F == MDH_F_MUL) {
+      if (p.redop == MDH_PW_ADD) T2_WARP(MDH_PW_ADD, MDH_F_MUL);
+      else if (p.redop == MDH_PW_MAX) T2_WARP(MDH_PW_MAX, MDH_F_MUL);
+      else T2_WARP(MDH_PW_MIN, MDH_F_MUL);
+    } else {
+      if (p.redop == MDH_PW_ADD) T2_WARP(MDH_PW_ADD, MDH_F_IDENTITY);
+      else if (p.redop == MDH_PW_MAX) T2_WARP(MDH_PW_MAX, MDH_F_IDENTITY);
+      else T2_WARP(MDH_PW_MIN, MDH_F_IDENTITY);
+    }
+#undef T2_WARP
+    return post_launch("t2_warp_kernel");
+  }
 #define T2_ROW(OP, FF) t2_row_kernel<TI, V, OP, FF><<<(unsigned)std::min<int64_t>(units, 148LL * 64), 256, 0, st>>>(P)
 #define T2_COL(OP, FF) t2_col_kernel<TI, V, OP, FF><<<(unsigned)std::min<int64_t>((units + 255) / 256, 148LL * 64), 256, 0, st>>>(P)
   if (row) {
@@ -357,9 +436,8 @@ mdh_status launch_t2(const Plan& p, const void* const* in, void* const* out, voi
   size_t part = (P.S > 1) ? (size_t)p.Ncc * P.S * compute_size(p) : 0;
   P.partials = ws;
   P.tickets = (unsigned*)((char*)ws + (part + 255) / 256 * 256);
-  if (P.S > 1 && p.tiles.vec == 1) {
-    MDH_CUDA(cudaMemsetAsync(P.tickets, 0, (size_t)p.Ncc * 4, st));
-  }
+  // the ticket words must be zero at entry: the workspace is zero-filled once by its
+  // owner (mdh.h contract) and the last CTA of every cc point resets its ticket
   switch (p.in[0].dtype) {
     case MDH_F32: return launch_typed<float, float>(p, P, st);
     case MDH_BF16: return launch_typed<uint16_t, float>(p, P, st);

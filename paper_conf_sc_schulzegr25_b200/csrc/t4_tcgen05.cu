@@ -253,11 +253,46 @@ __global__ void __launch_bounds__(THREADS, 1)
   }
 }
 
+// ---- operand normalisation pre-pass ---------------------------------------------------
+// An operand whose (MN, K) offsets are not 2-D linear (e.g. CCSD(T)'s t2 in output order,
+// the stride-2 im2col view of an MCC image) is gathered once per execute into a 2-D
+// K-major [MN][ld] (or MN-major [K][ld]) bf16 copy in the workspace; the GEMM then reads
+// it with TMA.  16-byte chunks when the source is contiguous along the inner dim.
+struct PermParams {
+  const uint16_t* src;
+  uint16_t* dst;
+  const int64_t* offO;   // outer-dim offsets (MN for K-major, K for MN-major)
+  const int64_t* offI;   // inner-dim offsets
+  int64_t nO, nI, ld;
+  int chunked;           // inner offsets contiguous in runs of 8 (aligned)
+};
+
+__global__ void __launch_bounds__(256) permute_kernel(const __grid_constant__ PermParams P) {
+  if (P.chunked) {
+    const int64_t nc = P.nI / 8;
+    const int64_t total = P.nO * nc;
+    for (int64_t e = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; e < total; e += (int64_t)gridDim.x * blockDim.x) {
+      const int64_t o = e / nc, c = e % nc;
+      const uint4 v = __ldg(reinterpret_cast<const uint4*>(P.src + P.offO[o] + P.offI[c * 8]));
+      *reinterpret_cast<uint4*>(P.dst + o * P.ld + c * 8) = v;
+    }
+  } else {
+    const int64_t total = P.nO * P.nI;
+    for (int64_t e = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; e < total; e += (int64_t)gridDim.x * blockDim.x) {
+      const int64_t o = e / P.nI, i = e % P.nI;
+      P.dst[o * P.ld + i] = P.src[P.offO[o] + __ldg(P.offI + i)];
+    }
+  }
+}
+
 // ------------------------------------------------------------------------- host
 struct Layout2D {
   bool ok = false;
   bool mn_major = false;       // unit stride along M (N) instead of K
   int64_t ld = 0;              // stride (elements) of the non-unit dim
+  bool permuted = false;       // gathered into the workspace by permute_kernel
+  int chunked = 0;
+  size_t ws_off = 0;
 };
 
 static bool linear(const std::vector<int64_t>& t, int64_t* stride) {
@@ -304,17 +339,54 @@ static Layout2D operand_layout(const Plan& p, const int* mdims, int nmd, int64_t
 
 }  // namespace t4
 
+// direct TMA operand, or a planned gather into a 2-D layout (operand normalisation)
+static t4::Layout2D plan_operand(const Plan& p, const int* mdims, int nmd, int64_t MN, const Access& acc,
+                                 std::string* why, const char* name, size_t* ws) {
+  t4::Layout2D L = t4::operand_layout(p, mdims, nmd, MN, acc, why, name);
+  if (L.ok && acc.base % 8 == 0) return L;
+  const Contraction& c = p.con;
+  std::vector<int64_t> tk = t4::table(p, c.kd, c.nk, acc), tm = t4::table(p, mdims, nmd, acc);
+  auto runs8 = [&](const std::vector<int64_t>& t) {
+    if (t.size() % 8) return false;
+    for (size_t i = 0; i < t.size(); i += 8) {
+      if ((t[i] + acc.base) % 8) return false;
+      for (int j = 1; j < 8; ++j)
+        if (t[i + j] != t[i] + j) return false;
+    }
+    return true;
+  };
+  L = t4::Layout2D();
+  L.ok = true;
+  L.permuted = true;
+  if (runs8(tk) || !runs8(tm)) {        // K-major copy [MN][ld]
+    L.mn_major = false;
+    L.ld = (c.K + 7) / 8 * 8;
+    L.chunked = runs8(tk);
+    *ws = (*ws + 255) / 256 * 256;
+    L.ws_off = *ws;
+    *ws += (size_t)MN * L.ld * 2;
+  } else {                              // MN-major copy [K][ld]
+    L.mn_major = true;
+    L.ld = (MN + 7) / 8 * 8;
+    L.chunked = 1;
+    *ws = (*ws + 255) / 256 * 256;
+    L.ws_off = *ws;
+    *ws += (size_t)c.K * L.ld * 2;
+  }
+  return L;
+}
+
 bool t4_supported(const Plan& p, std::string* why) {
   const Contraction& c = p.con;
   if (c.Z != 1) { *why = "batched contraction (Z>1) not in the tcgen05 template yet"; return false; }
   if (p.out[0].dtype != MDH_F32 && p.out[0].dtype != MDH_BF16) { *why = "output must be f32/bf16"; return false; }
-  if (p.in[c.a_buf].acc[0].base % 8 || p.in[c.b_buf].acc[0].base % 8) { *why = "operand base not 16-byte aligned"; return false; }
-  t4::Layout2D a = t4::operand_layout(p, c.md, c.nm, c.M, p.in[c.a_buf].acc[0], why, "A");
-  if (!a.ok) return false;
-  t4::Layout2D b = t4::operand_layout(p, c.nd, c.nn, c.N, p.in[c.b_buf].acc[0], why, "B");
-  if (!b.ok) return false;
   if (c.M > INT32_MAX || c.N > INT32_MAX || c.K > INT32_MAX) { *why = "extent exceeds TMA coordinates"; return false; }
-  *why = std::string("A ") + (a.mn_major ? "MN" : "K") + "-major, B " + (b.mn_major ? "MN" : "K") + "-major";
+  size_t ws = 0;
+  std::string w;
+  t4::Layout2D a = plan_operand(p, c.md, c.nm, c.M, p.in[c.a_buf].acc[0], &w, "A", &ws);
+  t4::Layout2D b = plan_operand(p, c.nd, c.nn, c.N, p.in[c.b_buf].acc[0], &w, "B", &ws);
+  *why = std::string("A ") + (a.permuted ? "gathered " : "") + (a.mn_major ? "MN" : "K") + "-major, B " +
+         (b.permuted ? "gathered " : "") + (b.mn_major ? "MN" : "K") + "-major";
   return true;
 }
 
@@ -328,8 +400,9 @@ mdh_status prepare_t4(Plan* p) {
   if (!t4_supported(*p, &why)) { set_error("T4: %s", why.c_str()); return MDH_ERR_UNSUPPORTED; }
   const Contraction& c = p->con;
   T4State* s = new T4State();
-  s->a = t4::operand_layout(*p, c.md, c.nm, c.M, p->in[c.a_buf].acc[0], &why, "A");
-  s->b = t4::operand_layout(*p, c.nd, c.nn, c.N, p->in[c.b_buf].acc[0], &why, "B");
+  size_t ws = 0;
+  s->a = plan_operand(*p, c.md, c.nm, c.M, p->in[c.a_buf].acc[0], &why, "A", &ws);
+  s->b = plan_operand(*p, c.nd, c.nn, c.N, p->in[c.b_buf].acc[0], &why, "B", &ws);
   int64_t akc, bkc;
   p->host_const.clear();
   build_contraction_tables(p, &akc, &bkc);
@@ -358,8 +431,8 @@ mdh_status prepare_t4(Plan* p) {
   P.ldc = sm;
   P.cbase = p->out[0].acc[0].base;
   p->tmaps = s;
-  p->t4_variant = 1;
-  p->ws_kernel = 0;
+  p->t4_variant = 1 + (s->a.permuted ? 2 : 0) + (s->b.permuted ? 4 : 0);
+  p->ws_kernel = ws;
   p->tiles.bm = t4::BM;
   p->tiles.bn = t4::BN;
   p->tiles.bk = t4::BK;
@@ -403,7 +476,23 @@ static mdh_status make_map(CUtensorMap* map, const void* base, int64_t inner, in
   return MDH_OK;
 }
 
-mdh_status launch_t4(const Plan& p, const void* const* in, void* const* out, void*, cudaStream_t st) {
+static mdh_status run_permute(const t4::Layout2D& L, const uint16_t* src, char* ws, const int64_t* offMN,
+                              const int64_t* offK, int64_t MN, int64_t K, cudaStream_t st, const uint16_t** out) {
+  t4::PermParams Q;
+  Q.src = src;
+  Q.dst = (uint16_t*)(ws + L.ws_off);
+  Q.ld = L.ld;
+  Q.chunked = L.chunked;
+  if (L.mn_major) { Q.offO = offK; Q.offI = offMN; Q.nO = K; Q.nI = MN; }
+  else { Q.offO = offMN; Q.offI = offK; Q.nO = MN; Q.nI = K; }
+  const int64_t work = Q.chunked ? Q.nO * (Q.nI / 8) : Q.nO * Q.nI;
+  const unsigned g = (unsigned)std::max<int64_t>(1, std::min<int64_t>((work + 255) / 256, 148LL * 32));
+  t4::permute_kernel<<<g, 256, 0, st>>>(Q);
+  *out = Q.dst;
+  return post_launch("t4_permute_kernel");
+}
+
+mdh_status launch_t4(const Plan& p, const void* const* in, void* const* out, void* ws, cudaStream_t st) {
   const char* dc = nullptr;
   MDH_TRY(device_consts(p, &dc));
   const T4State* s = (const T4State*)p.tmaps;
@@ -414,6 +503,12 @@ mdh_status launch_t4(const Plan& p, const void* const* in, void* const* out, voi
   P.cN = (const int64_t*)(dc + p.tab_off[5]);
   const uint16_t* A = (const uint16_t*)in[c.a_buf] + p.in[c.a_buf].acc[0].base;
   const uint16_t* B = (const uint16_t*)in[c.b_buf] + p.in[c.b_buf].acc[0].base;
+  if (s->a.permuted)
+    MDH_TRY(run_permute(s->a, A, (char*)ws, (const int64_t*)(dc + p.tab_off[0]), (const int64_t*)(dc + p.tab_off[1]),
+                        c.M, c.K, st, &A));
+  if (s->b.permuted)
+    MDH_TRY(run_permute(s->b, B, (char*)ws, (const int64_t*)(dc + p.tab_off[2]), (const int64_t*)(dc + p.tab_off[3]),
+                        c.N, c.K, st, &B));
   CUtensorMap ma, mb;
   if (s->a.mn_major) MDH_TRY(make_map(&ma, A, c.M, c.K, s->a.ld, 64, 64));
   else MDH_TRY(make_map(&ma, A, c.K, c.M, s->a.ld, 64, 128));

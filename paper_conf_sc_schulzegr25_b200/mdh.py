@@ -236,7 +236,8 @@ class Plan:
         import torch
         if self._ws is None or self._ws.numel() < self.workspace_bytes + 256:
             dev = device if device is not None else torch.device("cuda", self.device_index)
-            self._ws = torch.empty(self.workspace_bytes + 256, dtype=torch.uint8, device=dev)
+            # zero-filled once (mdh.h workspace contract); executes keep it consistent
+            self._ws = torch.zeros(self.workspace_bytes + 256, dtype=torch.uint8, device=dev)
         p = self._ws.data_ptr()
         return (p + 255) // 256 * 256
 

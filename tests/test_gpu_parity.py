@@ -367,3 +367,32 @@ def test_matmul_bf16_full_size():
     x = G.matmul_inputs(4096, 4096, 4096, "bf16", "identity")
     got, _ = run_gpu(spec, x)
     assert np.array_equal(got[0], G.bf16_bits_to_f32(x[1]))
+
+
+def test_ccsd_bf16_tcgen05():
+    # tiny brute-force size, the paper's Inp.1 reading (C-22), then the O=24/V=72 config sampled
+    for spec, n in ((S.ccsd_sd1(2, 3, "bf16"), None), (S.ccsd_sd2(dtype="bf16"), 20000),
+                    (S.ccsd_sd1(24, 72, "bf16"), 20000)):
+        x = G.gen_inputs(spec, 4010)
+        got, p = run_gpu(spec, x)
+        assert p.template == "T4_tcgen05_contraction"
+        if n is None:
+            assert_close_full(spec, x, got, 1e-2, kind="scale")
+        else:
+            assert_close_points(spec, x, got, 1e-2, n=n, kind="scale")
+
+
+@pytest.mark.parametrize("cfg", [(2, 3, 4, 16, 3, 3, 8), (1, 7, 7, 512, 3, 3, 512), (1, 112, 112, 64, 7, 7, 3)])
+def test_mcc_bf16_tcgen05(cfg):
+    spec = S.mcc(*cfg, dtype="bf16")
+    x = G.mcc_inputs(spec)
+    got, p = run_gpu(spec, x)
+    assert p.template == "T4_tcgen05_contraction"
+    assert_close_full(spec, x, got, 1e-2, kind="scale")
+
+
+def test_mcc_bf16_config_sampled():
+    spec = S.mcc(256, 7, 7, 512, 3, 3, 512, "bf16")
+    x = G.mcc_inputs(spec)
+    got, _ = run_gpu(spec, x)
+    assert_close_points(spec, x, got, 1e-2, n=5000, kind="scale")
