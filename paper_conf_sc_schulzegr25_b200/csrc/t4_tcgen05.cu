@@ -32,7 +32,7 @@ void build_contraction_tables(Plan* p, int64_t* a_kc, int64_t* b_kc);
 namespace t4 {
 
 constexpr int BM = 128, BN = 256, BK = 64, STAGES = 4;
-constexpr int THREADS = 192;
+constexpr int THREADS = 320;                 // 2 control warps + 8 epilogue warps
 constexpr int A_BYTES = BM * BK * 2;          // 16 KB
 constexpr int B_BYTES = BN * BK * 2;          // 32 KB
 constexpr int STAGE_BYTES = A_BYTES + B_BYTES;
@@ -50,7 +50,25 @@ struct Params {
   int64_t ldc, cbase;
   const int64_t* cM;                // generic output tables
   const int64_t* cN;
+  int sched;                        // 0: round-robin, M-major; 1: contiguous range per CTA, N-major
 };
+
+// Tile schedule shared by the three roles.  Round-robin M-major keeps concurrently running
+// CTAs on neighbouring tiles (operand reuse in L2); the contiguous N-major range keeps one
+// CTA on the same N-tile for many consecutive tiles, so the scatter epilogue caches that
+// tile's column offsets in shared memory.
+__device__ __forceinline__ int t_first(const Params& P) {
+  return P.sched ? (int)((int64_t)blockIdx.x * P.num_tiles / gridDim.x) : (int)blockIdx.x;
+}
+__device__ __forceinline__ int t_last(const Params& P) {
+  return P.sched ? (int)((int64_t)(blockIdx.x + 1) * P.num_tiles / gridDim.x) : P.num_tiles;
+}
+__device__ __forceinline__ int t_step(const Params& P) { return P.sched ? 1 : (int)gridDim.x; }
+__device__ __forceinline__ void t_decode(const Params& P, int t, int* mb, int* nb) {
+  if (P.sched) { *nb = t / P.tiles_m; *mb = t % P.tiles_m; }
+  else { *mb = t / P.tiles_n; *nb = t % P.tiles_n; }
+}
+__device__ __forceinline__ void named_sync(int id, int n) { asm volatile("bar.sync %0, %1;" ::"r"(id), "r"(n) : "memory"); }
 
 __device__ __forceinline__ uint32_t smem_u32(const void* p) { return (uint32_t)__cvta_generic_to_shared(p); }
 
@@ -109,10 +127,12 @@ __device__ __forceinline__ void tmem_ld32(uint32_t taddr, uint32_t* r) {
   asm volatile("tcgen05.wait::ld.sync.aligned;" ::: "memory");
 }
 
+template <int EPI, bool OUT_BF16>
 __global__ void __launch_bounds__(THREADS, 1)
     gemm_kernel(const __grid_constant__ CUtensorMap mapA, const __grid_constant__ CUtensorMap mapB,
                 const __grid_constant__ Params P) {
   extern __shared__ __align__(1024) uint8_t smem_raw[];
+  __shared__ int64_t s_cn[BN];      // column offsets of the current N-tile (scatter epilogue)
   uint8_t* smem = (uint8_t*)(((uintptr_t)smem_raw + 1023) & ~(uintptr_t)1023);
   uint8_t* sA = smem;
   uint8_t* sB = smem + STAGES * A_BYTES;
@@ -132,7 +152,7 @@ __global__ void __launch_bounds__(THREADS, 1)
     }
     for (int a = 0; a < 2; ++a) {
       mbar_init(tfull0 + 8 * a, 1);
-      mbar_init(tempty0 + 8 * a, 128);
+      mbar_init(tempty0 + 8 * a, 256);
     }
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
   }
@@ -151,8 +171,10 @@ __global__ void __launch_bounds__(THREADS, 1)
       // ===== TMA producer =====
       int stage = 0;
       uint32_t phase = 0;
-      for (int t = blockIdx.x; t < P.num_tiles; t += gridDim.x) {
-        const int m0 = (t / P.tiles_n) * BM, n0 = (t % P.tiles_n) * BN;
+      for (int t = t_first(P); t < t_last(P); t += t_step(P)) {
+        int mb, nb;
+        t_decode(P, t, &mb, &nb);
+        const int m0 = mb * BM, n0 = nb * BN;
         for (int kb = 0; kb < P.num_kb; ++kb) {
           mbar_wait(empty0 + 8 * stage, phase ^ 1);
           const uint32_t fb = full0 + 8 * stage;
@@ -181,7 +203,7 @@ __global__ void __launch_bounds__(THREADS, 1)
       int stage = 0;
       uint32_t phase = 0;
       int it = 0;
-      for (int t = blockIdx.x; t < P.num_tiles; t += gridDim.x, ++it) {
+      for (int t = t_first(P); t < t_last(P); t += t_step(P), ++it) {
         const int acc = it & 1;
         mbar_wait(tempty0 + 8 * acc, ((it >> 1) & 1) ^ 1);
         tc_fence_after();
@@ -205,38 +227,67 @@ __global__ void __launch_bounds__(THREADS, 1)
       }
     }
   } else {
-    // ===== epilogue: warps 2..5 → TMEM lane quadrant (warp % 4) =====
+    // ===== epilogue: warps 2..9; warp → TMEM lane quadrant (warp % 4) and a half of the
+    // 256 accumulator columns (two warps per sub-partition hide the store latency) =====
     const int quad = warp & 3;
+    const int half = (warp - 2) >> 2;
     const int row = quad * 32 + lane;
     int it = 0;
-    for (int t = blockIdx.x; t < P.num_tiles; t += gridDim.x, ++it) {
+    int cached_nb = -1;
+    for (int t = t_first(P); t < t_last(P); t += t_step(P), ++it) {
       const int acc = it & 1;
-      const int64_t m = (int64_t)(t / P.tiles_n) * BM + row;
-      const int64_t n0 = (int64_t)(t % P.tiles_n) * BN;
+      int mb, nbk;
+      t_decode(P, t, &mb, &nbk);
+      const int64_t m = (int64_t)mb * BM + row;
+      const int64_t n0 = (int64_t)nbk * BN + half * (BN / 2);
+      if (EPI == 1 && nbk != cached_nb) {
+        // (re)load this N-tile's column offsets into shared memory (epilogue warps only)
+        const int et = threadIdx.x - 64;
+        named_sync(1, 256);
+        const int64_t nn = (int64_t)nbk * BN + et;
+        s_cn[et] = __ldg(P.cN + min(nn, P.N - 1));
+        named_sync(1, 256);
+        cached_nb = nbk;
+      }
       mbar_wait(tfull0 + 8 * acc, (it >> 1) & 1);
       tc_fence_after();
       const bool mok = m < P.M;
-      const int64_t crow = mok ? (P.c_rowmajor ? P.cbase + m * P.ldc : P.cbase + P.cM[m]) : 0;
+      const int64_t crow = P.cbase + (EPI == 0 ? (mok ? m : 0) * P.ldc : __ldg(P.cM + (mok ? m : 0)));
 #pragma unroll 1
-      for (int c = 0; c < BN / 32; ++c) {
+      for (int c = 0; c < BN / 64; ++c) {
         uint32_t r[32];
-        tmem_ld32(tmem + ((uint32_t)(quad * 32) << 16) + acc * BN + c * 32, r);
-        if (!mok) continue;
+        tmem_ld32(tmem + ((uint32_t)(quad * 32) << 16) + acc * BN + half * (BN / 2) + c * 32, r);
         const int64_t nb = n0 + c * 32;
-        if (P.c_rowmajor && !P.out_bf16 && nb + 32 <= P.N && ((crow + nb) & 3) == 0) {
-          float4* dst = reinterpret_cast<float4*>(P.C + crow + nb);
+        if (EPI == 0) {
+          // row-major fp32 C: each thread writes 128 contiguous bytes of its row
+          if (mok && nb + 32 <= P.N && ((crow + nb) & 3) == 0) {
+            float4* dst = reinterpret_cast<float4*>(P.C + crow + nb);
 #pragma unroll
-          for (int j = 0; j < 8; ++j)
-            dst[j] = make_float4(__uint_as_float(r[4 * j]), __uint_as_float(r[4 * j + 1]), __uint_as_float(r[4 * j + 2]),
-                                 __uint_as_float(r[4 * j + 3]));
+            for (int j = 0; j < 8; ++j)
+              dst[j] = make_float4(__uint_as_float(r[4 * j]), __uint_as_float(r[4 * j + 1]),
+                                   __uint_as_float(r[4 * j + 2]), __uint_as_float(r[4 * j + 3]));
+          } else if (mok) {
+#pragma unroll
+            for (int j = 0; j < 32; ++j)
+              if (nb + j < P.N) P.C[crow + nb + j] = __uint_as_float(r[j]);
+          }
         } else {
+          // scatter through the output tables: column offsets first (branch-free,
+          // clamped read-only loads), then the stores; lanes = consecutive rows, so a
+          // store instruction is coalesced when the output is contiguous along m
 #pragma unroll
-          for (int j = 0; j < 32; ++j) {
-            const int64_t n = nb + j;
-            if (n < P.N) {
-              const int64_t o = crow + (P.c_rowmajor ? n : P.cN[n]);
-              if (P.out_bf16) ((__nv_bfloat16*)P.C)[o] = __float2bfloat16_rn(__uint_as_float(r[j]));
-              else P.C[o] = __uint_as_float(r[j]);
+          for (int h = 0; h < 2; ++h) {
+            int64_t co[16];
+#pragma unroll
+            for (int j = 0; j < 16; ++j) co[j] = s_cn[half * (BN / 2) + c * 32 + h * 16 + j];
+#pragma unroll
+            for (int j = 0; j < 16; ++j) {
+              if (mok && nb + h * 16 + j < P.N) {
+                const int64_t o = crow + co[j];
+                const float v = __uint_as_float(r[h * 16 + j]);
+                if (OUT_BF16) ((__nv_bfloat16*)P.C)[o] = __float2bfloat16_rn(v);
+                else __stcs(P.C + o, v);
+              }
             }
           }
         }
@@ -430,6 +481,7 @@ mdh_status prepare_t4(Plan* p) {
   P.c_rowmajor = lm && ln && sn == 1 && cm[0] == 0 && cn[0] == 0;
   P.ldc = sm;
   P.cbase = p->out[0].acc[0].base;
+  P.sched = P.c_rowmajor ? 0 : 1;
   p->tmaps = s;
   p->t4_variant = 1 + (s->a.permuted ? 2 : 0) + (s->b.permuted ? 4 : 0);
   p->ws_kernel = ws;
@@ -517,14 +569,21 @@ mdh_status launch_t4(const Plan& p, const void* const* in, void* const* out, voi
   static std::once_flag attr_once;
   static cudaError_t attr_err = cudaSuccess;
   std::call_once(attr_once, [] {
-    attr_err = cudaFuncSetAttribute(t4::gemm_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, t4::SMEM_BYTES);
+    const void* ks[3] = {(const void*)t4::gemm_kernel<0, false>, (const void*)t4::gemm_kernel<1, false>,
+                         (const void*)t4::gemm_kernel<1, true>};
+    for (const void* k : ks) {
+      cudaError_t e = cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, t4::SMEM_BYTES);
+      if (e != cudaSuccess) attr_err = e;
+    }
   });
   MDH_CUDA(attr_err);
   int dev = 0, sms = 148;
   cudaGetDevice(&dev);
   cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
   const int grid = std::min(P.num_tiles, sms);
-  t4::gemm_kernel<<<grid, t4::THREADS, t4::SMEM_BYTES, st>>>(ma, mb, P);
+  if (P.c_rowmajor && !P.out_bf16) t4::gemm_kernel<0, false><<<grid, t4::THREADS, t4::SMEM_BYTES, st>>>(ma, mb, P);
+  else if (!P.out_bf16) t4::gemm_kernel<1, false><<<grid, t4::THREADS, t4::SMEM_BYTES, st>>>(ma, mb, P);
+  else t4::gemm_kernel<1, true><<<grid, t4::THREADS, t4::SMEM_BYTES, st>>>(ma, mb, P);
   return post_launch("t4_gemm_kernel");
 }
 

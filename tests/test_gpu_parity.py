@@ -347,11 +347,13 @@ def test_matmul_bf16_tcgen05(mnk, at, bt):
     spec = _mm_spec(M, N, K, at, bt)
     x = G.gen_inputs(spec, 3100, "positive")
     got, p = run_gpu(spec, x)
-    # TMA needs a 16-byte aligned leading dimension: A^T needs M%8==0, A needs K%8==0, etc.
+    # operands without a 16-byte aligned leading dimension are gathered into a TMA layout
+    d = p.describe()
     lda = M if at else K
     ldb = K if bt else N
-    tma_ok = lda % 8 == 0 and ldb % 8 == 0
-    assert p.template == ("T4_tcgen05_contraction" if tma_ok else "T3_simt_contraction"), p.describe()
+    assert p.template == "T4_tcgen05_contraction", d
+    assert (d["t4_variant"] & 2 != 0) == (lda % 8 != 0)
+    assert (d["t4_variant"] & 4 != 0) == (ldb % 8 != 0)
     assert_close_full(spec, x, got, 1e-2, kind="rel")
 
 

@@ -1,0 +1,45 @@
+"""Quick device timing of bench workloads (median of CUDA-event pairs, L2 flushed).
+
+    python tools/time_one.py ccsd_bf16 mcc_bf16 [--reps 10] [--force-tile split=4]
+"""
+import argparse
+import json
+import os
+import sys
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+sys.path.insert(0, ROOT)
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("workloads", nargs="+")
+    ap.add_argument("--reps", type=int, default=10)
+    ap.add_argument("--force-tile", default=None)
+    a = ap.parse_args()
+    import torch
+    import bench
+    from paper_conf_sc_schulzegr25_b200 import Plan, to_device
+    dev = torch.device("cuda", 0)
+    pk = bench.peaks()
+    flush = torch.empty(2 * torch.cuda.get_device_properties(dev).L2_cache_size // 4, device=dev)
+    for name in a.workloads:
+        w = bench.workload(name)
+        plan = Plan(w["spec"], force_tile=a.force_tile)
+        tin = [to_device(x, b["dtype"], dev) for x, b in zip(w["inputs"](), w["spec"]["inputs"])]
+        outs = plan.empty_outputs(dev)
+        for _ in range(3):
+            plan(tin, outs)
+        torch.cuda.synchronize()
+        ts = sorted(bench.time_steps(lambda: plan(tin, outs), a.reps, torch.cuda.current_stream(), flush))
+        med = ts[len(ts) // 2]
+        rl = bench.roofline(w, med, pk)
+        print(json.dumps({"workload": name, "template": plan.template, "ms": round(med * 1e3, 4),
+                          "value": round(w["work"] / med / w["scale"], 2), "unit": w["unit"],
+                          "frac": round(rl["frac"], 4), "tiles": plan.describe()["tiles"]}), flush=True)
+        del tin, outs, plan
+        torch.cuda.empty_cache()
+
+
+if __name__ == "__main__":
+    main()
