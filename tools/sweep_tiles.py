@@ -1,0 +1,108 @@
+"""Measured tile sweep on B200 → tiles/b200.json (replaces ATF).
+
+    python tools/sweep_tiles.py [--out tiles/b200.json] [--reps 15]
+
+For each (workload, candidate tile override) the step is timed with CUDA events (median of
+--reps, L2 flushed between reps); the best candidate per (template, dtype, shape bucket)
+is written as a table entry.  Every candidate's median is kept in the "sweep" record.
+"""
+import argparse
+import json
+import math
+import os
+import sys
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+sys.path.insert(0, ROOT)
+
+# (workload, spec builder kwargs, candidates)
+def cases():
+    from mdh_workloads import specs as S
+    from mdh_workloads import gen as G
+    return [
+        ("dot_f32_2^20", lambda: (S.dot(1 << 20, "f32"), G.dot_inputs(1 << 20, "f32")),
+         [f"split={s}" for s in (64, 128, 148, 256, 296, 512, 592, 1184)]),
+        ("dot_f32_2^24", lambda: (S.dot(1 << 24, "f32"), G.dot_inputs(1 << 24, "f32")),
+         [f"split={s}" for s in (296, 592, 1184, 2368)]),
+        ("dot_f32_2^28", lambda: (S.dot(1 << 28, "f32"), G.dot_inputs(1 << 28, "f32")),
+         [f"split={s}" for s in (592, 1184, 2368, 4736)]),
+        ("dot_i32_2^20", lambda: (S.dot(1 << 20, "i32"), G.dot_inputs(1 << 20, "i32")),
+         [f"split={s}" for s in (64, 128, 148, 256, 296, 512)]),
+        ("jacobi3d", lambda: (S.jacobi3d(512, 512, 512), G.jacobi3d_inputs(512, 512, 512)),
+         [f"zchunk={z}" for z in (8, 16, 32, 64, 128, 255, 510)]),
+        ("prl_B", lambda: (S.prl(1 << 14, 1 << 20), G.prl_inputs(1 << 14, 1 << 20)),
+         [f"split={s}" for s in (8, 16, 32, 37, 48, 64)]),
+        ("mcc_f32_n1", lambda: (S.mcc(1, 7, 7, 512, 3, 3, 512, "f32"),
+                                G.mcc_inputs(S.mcc(1, 7, 7, 512, 3, 3, 512, "f32"))),
+         [f"split={s}" for s in (1, 8, 16, 32, 64, 72)]),
+    ]
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--out", default=os.path.join(ROOT, "tiles", "b200.json"))
+    ap.add_argument("--reps", type=int, default=15)
+    ap.add_argument("--only", default=None)
+    a = ap.parse_args()
+    import torch
+    import bench
+    from paper_conf_sc_schulzegr25_b200 import Plan, to_device
+    dev = torch.device("cuda", 0)
+    flush = torch.empty(2 * torch.cuda.get_device_properties(dev).L2_cache_size // 4, device=dev)
+    table = json.load(open(a.out)) if os.path.exists(a.out) else {"entries": []}
+    entries = {(e["template"], e["dtype"], tuple(e["bucket"])): e for e in table.get("entries", [])}
+    log = []
+    for name, mk, cands in cases():
+        if a.only and a.only not in name:
+            continue
+        spec, host = mk()
+        tin = None
+        res = []
+        for c in [None] + cands:
+            plan = Plan(spec, force_tile=c) if c else Plan(spec)
+            if tin is None:
+                tin = [to_device(x, b["dtype"], dev) for x, b in zip(host, spec["inputs"])]
+            outs = plan.empty_outputs(dev)
+            ws = plan.workspace(dev) if plan.workspace_bytes else None
+            step = lambda: plan(tin, outs, workspace_ptr=ws)
+            for _ in range(3):
+                step()
+            torch.cuda.synchronize()
+            ts = sorted(bench.time_steps(step, a.reps, torch.cuda.current_stream(), flush))
+            med = ts[len(ts) // 2]
+            d = plan.describe()
+            res.append((med, c, d))
+            print(json.dumps({"workload": name, "cand": c or "default", "us": round(med * 1e6, 2),
+                              "template": d["template"], "tiles": d["tiles"]}), flush=True)
+        best = min(res, key=lambda r: r[0])
+        d = best[2]
+        if d["template"] in ("T3_simt_contraction", "T4_tcgen05_contraction"):
+            c = d["contraction"]
+            bucket = [round(math.log2(c["M"]), 2), round(math.log2(c["N"]), 2), round(math.log2(c["K"] * c["Z"]), 2)]
+        else:
+            bucket = [round(math.log2(d["Ncc"]), 2), round(math.log2(d["Nred"]), 2)]
+        dtype = spec["inputs"][0]["dtype"]
+        tiles = {}
+        if best[1]:
+            for kv in best[1].split(","):
+                k, v = kv.split("=")
+                tiles[k] = int(v)
+        key = (d["template"], dtype, tuple(bucket))
+        entries[key] = {"template": d["template"], "dtype": dtype, "bucket": bucket, "tiles": tiles,
+                        "workload": name, "median_us": round(best[0] * 1e6, 2),
+                        "default_us": round(res[0][0] * 1e6, 2),
+                        "sweep": {(r[1] or "default"): round(r[0] * 1e6, 2) for r in res}}
+        log.append(entries[key])
+        del tin
+        torch.cuda.empty_cache()
+    table["entries"] = sorted(entries.values(), key=lambda e: (e["template"], e["dtype"], e["bucket"]))
+    table["comment"] = ("Tile table for libmdh on B200 (sm_100a), produced by tools/sweep_tiles.py: median CUDA-event "
+                        "time of every candidate (L2 flushed), best per (template, dtype, log2 shape bucket). "
+                        "An entry with empty tiles means the planner default won.")
+    with open(a.out, "w") as f:
+        json.dump(table, f, indent=1)
+    print("wrote", a.out, len(table["entries"]), "entries")
+
+
+if __name__ == "__main__":
+    main()
