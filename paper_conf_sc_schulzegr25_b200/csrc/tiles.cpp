@@ -183,7 +183,9 @@ void lookup_tiles(Plan* p, const char* table_path, const char* force) {
       if (d < bestd) { bestd = d; best = &e; }
     }
   }
-  if (best) {
+  // a measured entry more than 6 octaves (summed log2 distance) away says nothing about
+  // this shape: keep the template defaults then
+  if (best && bestd <= 6.0) {
     const J* tl = best->get("tiles");
     if (tl)
       for (auto& kv : tl->obj) apply(&t, kv.first, kv.second.num);

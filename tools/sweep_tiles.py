@@ -48,7 +48,7 @@ def main():
     import bench
     from paper_conf_sc_schulzegr25_b200 import Plan, to_device
     dev = torch.device("cuda", 0)
-    flush = torch.empty(2 * torch.cuda.get_device_properties(dev).L2_cache_size // 4, device=dev)
+    flush = bench.L2Flush(dev)
     table = json.load(open(a.out)) if os.path.exists(a.out) else {"entries": []}
     entries = {(e["template"], e["dtype"], tuple(e["bucket"])): e for e in table.get("entries", [])}
     log = []

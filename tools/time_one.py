@@ -22,7 +22,7 @@ def main():
     from paper_conf_sc_schulzegr25_b200 import Plan, to_device
     dev = torch.device("cuda", 0)
     pk = bench.peaks()
-    flush = torch.empty(2 * torch.cuda.get_device_properties(dev).L2_cache_size // 4, device=dev)
+    flush = bench.L2Flush(dev)
     for name in a.workloads:
         w = bench.workload(name)
         plan = Plan(w["spec"], force_tile=a.force_tile)
