@@ -170,7 +170,7 @@ class L2Flush:
     def zero_(self):
         import torch
         self.w.zero_()
-        torch.sum(self.r, out=self.sink)
+        torch.sum(self.r, dim=0, out=self.sink)
 
 
 def time_steps(step, K, stream, flush):

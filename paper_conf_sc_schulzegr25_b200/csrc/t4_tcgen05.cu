@@ -296,11 +296,209 @@ __global__ void __launch_bounds__(THREADS, 1)
       mbar_arrive(tempty0 + 8 * acc);
     }
   }
+  __syncwarp();                  // lanes 1..31 of warps 0/1 wait for their role lane
   tc_fence_before();
   __syncthreads();
   if (warp == 1) {
     tc_fence_after();
     asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" ::"r"(tmem), "r"(TMEM_COLS));
+  }
+}
+
+// ---- 2-SM variant: a CTA pair (cluster 2×1) computes a 256×256 tile with
+// tcgen05.mma.cta_group::2 (M = 256 split over the two SMs' TMEM, each SM staging half of A
+// and half of B), so each SM streams 32 KB instead of 48 KB of operands per 64-deep k-block
+// for the same MMA work.  Barriers: the leader's full barrier counts both producers and
+// both CTAs' TMA bytes (cta_group::2 TMA signals the leader); MMA commits are multicast to
+// both CTAs' empty / tmem-full barriers; both epilogues release the accumulator at the
+// leader's tmem-empty barrier.
+constexpr int S2 = 6;                          // stages (32 KB each)
+constexpr int A2_BYTES = 128 * BK * 2;         // this CTA's half of A (16 KB)
+constexpr int B2_BYTES = 128 * BK * 2;         // this CTA's half of B (16 KB)
+constexpr int STAGE2_BYTES = A2_BYTES + B2_BYTES;
+constexpr int SMEM2_BYTES = S2 * STAGE2_BYTES + 1024 + 256;
+
+__device__ __forceinline__ uint32_t cluster_rank() {
+  uint32_t r;
+  asm volatile("mov.u32 %0, %%cluster_ctarank;" : "=r"(r));
+  return r;
+}
+__device__ __forceinline__ uint32_t map_to_rank0(uint32_t addr) {
+  uint32_t r;
+  asm volatile("mapa.shared::cluster.u32 %0, %1, 0;" : "=r"(r) : "r"(addr));
+  return r;
+}
+__device__ __forceinline__ void cluster_sync_all() {
+  asm volatile("barrier.cluster.arrive.release.aligned;\n\tbarrier.cluster.wait.acquire.aligned;" ::: "memory");
+}
+__device__ __forceinline__ void tma_load_2d_cg2(uint32_t dst, const CUtensorMap* map, uint32_t bar_cluster, int c0, int c1) {
+  asm volatile(
+      "cp.async.bulk.tensor.2d.cta_group::2.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1, {%3, %4}], [%2];" ::"r"(dst),
+      "l"((uint64_t)map), "r"(bar_cluster), "r"(c0), "r"(c1)
+      : "memory");
+}
+__device__ __forceinline__ void mma_bf16_cg2(uint32_t d_tmem, uint64_t a, uint64_t b, uint32_t idesc, uint32_t acc) {
+  asm volatile(
+      "{\n\t.reg .pred p;\n\tsetp.ne.b32 p, %4, 0;\n\t"
+      "tcgen05.mma.cta_group::2.kind::f16 [%0], %1, %2, %3, p;\n\t}" ::"r"(d_tmem),
+      "l"(a), "l"(b), "r"(idesc), "r"(acc));
+}
+__device__ __forceinline__ void mma_commit_cg2(uint32_t bar) {
+  asm volatile(
+      "{\n\t.reg .b16 m;\n\tmov.b16 m, 3;\n\t"
+      "tcgen05.commit.cta_group::2.mbarrier::arrive::one.shared::cluster.multicast::cluster.b64 [%0], m;\n\t}" ::"r"(bar)
+      : "memory");
+}
+__device__ __forceinline__ void mbar_arrive_cluster(uint32_t bar_cluster) {
+  asm volatile("mbarrier.arrive.release.cluster.shared::cluster.b64 _, [%0];" ::"r"(bar_cluster) : "memory");
+}
+
+template <bool OUT_ROWMAJOR>
+__global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(THREADS, 1)
+    gemm2_kernel(const __grid_constant__ CUtensorMap mapA, const __grid_constant__ CUtensorMap mapB,
+                 const __grid_constant__ Params P) {
+  extern __shared__ __align__(1024) uint8_t smem_raw[];
+  uint8_t* smem = (uint8_t*)(((uintptr_t)smem_raw + 1023) & ~(uintptr_t)1023);
+  uint8_t* sA = smem;
+  uint8_t* sB = smem + S2 * A2_BYTES;
+  uint64_t* bars = (uint64_t*)(smem + S2 * STAGE2_BYTES);
+  uint32_t* tmem_slot = (uint32_t*)(bars + 2 * S2 + 4);
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  const uint32_t rank = cluster_rank();
+  const bool leader = rank == 0;
+  const uint32_t full0 = smem_u32(bars), empty0 = smem_u32(bars + S2);
+  const uint32_t tfull0 = smem_u32(bars + 2 * S2), tempty0 = smem_u32(bars + 2 * S2 + 2);
+  // pair tiles: tiles_m/tiles_n count 256×256 tiles; clusters stride over them
+  const int cluster_id = blockIdx.x >> 1, nclusters = gridDim.x >> 1;
+
+  if (warp == 0 && lane == 0) {
+    asm volatile("prefetch.tensormap [%0];" ::"l"((uint64_t)&mapA) : "memory");
+    asm volatile("prefetch.tensormap [%0];" ::"l"((uint64_t)&mapB) : "memory");
+    for (int s = 0; s < S2; ++s) {
+      mbar_init(full0 + 8 * s, 2);
+      mbar_init(empty0 + 8 * s, 1);
+    }
+    for (int a = 0; a < 2; ++a) {
+      mbar_init(tfull0 + 8 * a, 1);
+      mbar_init(tempty0 + 8 * a, 16);          // 8 epilogue warps × 2 CTAs
+    }
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+  }
+  if (warp == 1) {
+    asm volatile("tcgen05.alloc.cta_group::2.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(smem_u32(tmem_slot)),
+                 "r"(TMEM_COLS));
+    asm volatile("tcgen05.relinquish_alloc_permit.cta_group::2.sync.aligned;");
+  }
+  tc_fence_before();
+  cluster_sync_all();
+  tc_fence_after();
+  const uint32_t tmem = *tmem_slot;
+
+  if (warp == 0) {
+    if (lane == 0) {
+      // ===== TMA producer (both CTAs; bytes are counted at the leader's full barrier) =====
+      int stage = 0;
+      uint32_t phase = 0;
+      for (int t = cluster_id; t < P.num_tiles; t += nclusters) {
+        const int m0 = (t / P.tiles_n) * 256 + (int)rank * 128, n0 = (t % P.tiles_n) * 256 + (int)rank * 128;
+        for (int kb = 0; kb < P.num_kb; ++kb) {
+          mbar_wait(empty0 + 8 * stage, phase ^ 1);
+          const uint32_t fb_leader = map_to_rank0(full0 + 8 * stage);
+          if (leader) mbar_expect_tx(full0 + 8 * stage, 2 * STAGE2_BYTES);
+          else mbar_arrive_cluster(fb_leader);
+          const uint32_t a_dst = smem_u32(sA + stage * A2_BYTES), b_dst = smem_u32(sB + stage * B2_BYTES);
+          const int k0 = kb * BK;
+          if (P.a_mn_major) {
+            tma_load_2d_cg2(a_dst, &mapA, fb_leader, m0, k0);
+            tma_load_2d_cg2(a_dst + 8192, &mapA, fb_leader, m0 + 64, k0);
+          } else {
+            tma_load_2d_cg2(a_dst, &mapA, fb_leader, k0, m0);
+          }
+          if (P.b_mn_major) {
+            tma_load_2d_cg2(b_dst, &mapB, fb_leader, n0, k0);
+            tma_load_2d_cg2(b_dst + 8192, &mapB, fb_leader, n0 + 64, k0);
+          } else {
+            tma_load_2d_cg2(b_dst, &mapB, fb_leader, k0, n0);
+          }
+          if (++stage == S2) { stage = 0; phase ^= 1; }
+        }
+      }
+    }
+  } else if (warp == 1) {
+    if (lane == 0 && leader) {
+      // ===== MMA issuer: leader CTA only, one thread, M=256 × N=256 per instruction =====
+      int stage = 0;
+      uint32_t phase = 0;
+      int it = 0;
+      for (int t = cluster_id; t < P.num_tiles; t += nclusters, ++it) {
+        const int acc = it & 1;
+        mbar_wait(tempty0 + 8 * acc, ((it >> 1) & 1) ^ 1);
+        tc_fence_after();
+        const uint32_t d = tmem + acc * BN;
+        for (int kb = 0; kb < P.num_kb; ++kb) {
+          mbar_wait(full0 + 8 * stage, phase);
+          tc_fence_after();
+          const uint32_t a0 = smem_u32(sA + stage * A2_BYTES), b0 = smem_u32(sB + stage * B2_BYTES);
+#pragma unroll
+          for (int k = 0; k < BK / 16; ++k) {
+            const uint64_t ad = P.a_mn_major ? sdesc(a0 + 2048 * k, 8192, 1024) : sdesc(a0 + 32 * k, 16, 1024);
+            const uint64_t bd = P.b_mn_major ? sdesc(b0 + 2048 * k, 8192, 1024) : sdesc(b0 + 32 * k, 16, 1024);
+            mma_bf16_cg2(d, ad, bd, P.idesc, (kb | k) != 0);
+          }
+          mma_commit_cg2(empty0 + 8 * stage);
+          if (++stage == S2) { stage = 0; phase ^= 1; }
+        }
+        mma_commit_cg2(tfull0 + 8 * acc);
+      }
+      // drain: the last accumulators must be released before the barriers go away
+      for (int k = 0; k < 2 && it - 1 - k >= 0; ++k) {
+        const int j = it - 1 - k;
+        mbar_wait(tempty0 + 8 * (j & 1), (j >> 1) & 1);
+      }
+    }
+  } else {
+    // ===== epilogue (both CTAs): this CTA's 128 accumulator rows =====
+    const int quad = warp & 3;
+    const int half = (warp - 2) >> 2;
+    const int row = quad * 32 + lane;
+    const uint32_t tempty_leader = map_to_rank0(tempty0);
+    int it = 0;
+    for (int t = cluster_id; t < P.num_tiles; t += nclusters, ++it) {
+      const int acc = it & 1;
+      const int64_t m = (int64_t)(t / P.tiles_n) * 256 + rank * 128 + row;
+      const int64_t n0 = (int64_t)(t % P.tiles_n) * 256 + half * 128;
+      mbar_wait(tfull0 + 8 * acc, (it >> 1) & 1);
+      tc_fence_after();
+      const bool mok = m < P.M;
+      const int64_t crow = P.cbase + (OUT_ROWMAJOR ? (mok ? m : 0) * P.ldc : __ldg(P.cM + (mok ? m : 0)));
+#pragma unroll 1
+      for (int c = 0; c < 4; ++c) {
+        uint32_t r[32];
+        tmem_ld32(tmem + ((uint32_t)(quad * 32) << 16) + acc * BN + half * 128 + c * 32, r);
+        const int64_t nb = n0 + c * 32;
+        if (OUT_ROWMAJOR && mok && nb + 32 <= P.N && ((crow + nb) & 3) == 0) {
+          float4* dst = reinterpret_cast<float4*>(P.C + crow + nb);
+#pragma unroll
+          for (int j = 0; j < 8; ++j)
+            dst[j] = make_float4(__uint_as_float(r[4 * j]), __uint_as_float(r[4 * j + 1]), __uint_as_float(r[4 * j + 2]),
+                                 __uint_as_float(r[4 * j + 3]));
+        } else if (mok) {
+#pragma unroll
+          for (int j = 0; j < 32; ++j)
+            if (nb + j < P.N) P.C[crow + (OUT_ROWMAJOR ? nb + j : __ldg(P.cN + nb + j))] = __uint_as_float(r[j]);
+        }
+      }
+      tc_fence_before();
+      __syncwarp();
+      if (lane == 0) mbar_arrive_cluster(tempty_leader + 8 * acc);
+    }
+  }
+  __syncwarp();                  // lanes 1..31 of warps 0/1 wait for their role lane
+  tc_fence_before();
+  asm volatile("barrier.cluster.arrive.release;\n\tbarrier.cluster.wait.acquire;" ::: "memory");
+  if (warp == 1) {
+    tc_fence_after();
+    asm volatile("tcgen05.dealloc.cta_group::2.sync.aligned.b32 %0, %1;" ::"r"(tmem), "r"(TMEM_COLS));
   }
 }
 
@@ -444,6 +642,7 @@ bool t4_supported(const Plan& p, std::string* why) {
 struct T4State {
   t4::Layout2D a, b;
   t4::Params P;
+  int cg = 1;      // 1: one SM per 128×256 tile; 2: SM pair per 256×256 tile
 };
 
 mdh_status prepare_t4(Plan* p) {
@@ -482,13 +681,23 @@ mdh_status prepare_t4(Plan* p) {
   P.ldc = sm;
   P.cbase = p->out[0].acc[0].base;
   P.sched = P.c_rowmajor ? 0 : 1;
+  // 2-SM pairs (cta_group::2, 256×256 tiles) for large row-major outputs when requested
+  // (tile knob cluster=2); measured slower than the 1-SM kernel so far
+  s->cg = (P.c_rowmajor && !P.out_bf16 && c.M >= 256 && c.N >= 256 && p->tiles.cluster == 2) ? 2 : 1;
+  if (s->cg == 2) {
+    P.tiles_m = (int)((c.M + 255) / 256);
+    P.tiles_n = (int)((c.N + 255) / 256);
+    P.num_tiles = P.tiles_m * P.tiles_n;
+    P.idesc = (P.idesc & ~(0x1Fu << 24)) | ((uint32_t)(256 >> 4) << 24);
+  }
   p->tmaps = s;
-  p->t4_variant = 1 + (s->a.permuted ? 2 : 0) + (s->b.permuted ? 4 : 0);
+  p->t4_variant = 1 + (s->a.permuted ? 2 : 0) + (s->b.permuted ? 4 : 0) + (s->cg == 2 ? 8 : 0);
   p->ws_kernel = ws;
-  p->tiles.bm = t4::BM;
+  p->tiles.bm = s->cg == 2 ? 256 : t4::BM;
   p->tiles.bn = t4::BN;
   p->tiles.bk = t4::BK;
-  p->tiles.stages = t4::STAGES;
+  p->tiles.stages = s->cg == 2 ? t4::S2 : t4::STAGES;
+  p->tiles.cluster = s->cg;
   return MDH_OK;
 }
 
@@ -565,7 +774,7 @@ mdh_status launch_t4(const Plan& p, const void* const* in, void* const* out, voi
   if (s->a.mn_major) MDH_TRY(make_map(&ma, A, c.M, c.K, s->a.ld, 64, 64));
   else MDH_TRY(make_map(&ma, A, c.K, c.M, s->a.ld, 64, 128));
   if (s->b.mn_major) MDH_TRY(make_map(&mb, B, c.N, c.K, s->b.ld, 64, 64));
-  else MDH_TRY(make_map(&mb, B, c.K, c.N, s->b.ld, 64, 256));
+  else MDH_TRY(make_map(&mb, B, c.K, c.N, s->b.ld, 64, s->cg == 2 ? 128 : 256));
   static std::once_flag attr_once;
   static cudaError_t attr_err = cudaSuccess;
   std::call_once(attr_once, [] {
@@ -575,11 +784,21 @@ mdh_status launch_t4(const Plan& p, const void* const* in, void* const* out, voi
       cudaError_t e = cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, t4::SMEM_BYTES);
       if (e != cudaSuccess) attr_err = e;
     }
+    const void* k2[2] = {(const void*)t4::gemm2_kernel<true>, (const void*)t4::gemm2_kernel<false>};
+    for (const void* k : k2) {
+      cudaError_t e = cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, t4::SMEM2_BYTES);
+      if (e != cudaSuccess) attr_err = e;
+    }
   });
   MDH_CUDA(attr_err);
   int dev = 0, sms = 148;
   cudaGetDevice(&dev);
   cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+  if (s->cg == 2) {
+    const int grid2 = 2 * std::min(P.num_tiles, sms / 2);
+    t4::gemm2_kernel<true><<<grid2, t4::THREADS, t4::SMEM2_BYTES, st>>>(ma, mb, P);
+    return post_launch("t4_gemm2_kernel");
+  }
   const int grid = std::min(P.num_tiles, sms);
   if (P.c_rowmajor && !P.out_bf16) t4::gemm_kernel<0, false><<<grid, t4::THREADS, t4::SMEM_BYTES, st>>>(ma, mb, P);
   else if (!P.out_bf16) t4::gemm_kernel<1, false><<<grid, t4::THREADS, t4::SMEM_BYTES, st>>>(ma, mb, P);
