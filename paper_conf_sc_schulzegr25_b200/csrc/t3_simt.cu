@@ -145,6 +145,104 @@ __global__ void __launch_bounds__(256, 1) t3_kernel(const __grid_constant__ T3Pa
   }
 }
 
+// ---- linear fast path (A[m·lda + k], B[k·ldb + n], C[m·ldc + n], fp32, 16-B aligned) ----
+// Same 128×128×8 tiling with float4 global loads, float4 shared-memory reads and float4
+// stores, no offset tables, ≤128 registers so two CTAs share an SM.
+struct T3Lin {
+  const float* A;
+  const float* B;
+  float* C;
+  int M, N, K, lda, ldb, ldc;
+};
+
+__global__ void __launch_bounds__(256, 2) t3_linear_kernel(const __grid_constant__ T3Lin P) {
+  __shared__ __align__(16) float As[2][8][128 + 4];
+  __shared__ __align__(16) float Bs[2][8][128];
+  const int tid = threadIdx.x, tx = tid & 15, ty = tid >> 4;
+  const int m0 = blockIdx.y * 128, n0 = blockIdx.x * 128;
+  const int am = tid >> 1, ak = (tid & 1) * 4;      // A: row am, 4 consecutive k
+  const int bk = tid >> 5, bn = (tid & 31) * 4;     // B: row bk, 4 consecutive n
+  const bool arow = m0 + am < P.M, bcol = n0 + bn + 3 < P.N;
+  const float* Ap = P.A + (int64_t)(m0 + am) * P.lda + ak;
+  const float* Bp = P.B + (int64_t)bk * P.ldb + n0 + bn;
+  float4 ra, rb;
+  auto gload = [&](int k0) {
+    ra = make_float4(0.f, 0.f, 0.f, 0.f);
+    rb = ra;
+    if (arow) {
+      if (k0 + ak + 3 < P.K) ra = __ldg(reinterpret_cast<const float4*>(Ap + k0));
+      else {
+        float t[4];
+        for (int j = 0; j < 4; ++j) t[j] = (k0 + ak + j < P.K) ? __ldg(Ap + k0 + j) : 0.f;
+        ra = make_float4(t[0], t[1], t[2], t[3]);
+      }
+    }
+    if (k0 + bk < P.K) {
+      const float* b = Bp + (int64_t)k0 * P.ldb;
+      if (bcol) rb = __ldg(reinterpret_cast<const float4*>(b));
+      else {
+        float t[4];
+        for (int j = 0; j < 4; ++j) t[j] = (n0 + bn + j < P.N) ? __ldg(b + j) : 0.f;
+        rb = make_float4(t[0], t[1], t[2], t[3]);
+      }
+    }
+  };
+  auto sstore = [&](int buf) {
+    As[buf][ak + 0][am] = ra.x;
+    As[buf][ak + 1][am] = ra.y;
+    As[buf][ak + 2][am] = ra.z;
+    As[buf][ak + 3][am] = ra.w;
+    *reinterpret_cast<float4*>(&Bs[buf][bk][bn]) = rb;
+  };
+  float acc[8][8];
+#pragma unroll
+  for (int i = 0; i < 8; ++i)
+#pragma unroll
+    for (int j = 0; j < 8; ++j) acc[i][j] = 0.f;
+  gload(0);
+  sstore(0);
+  __syncthreads();
+  int buf = 0;
+  for (int k0 = 0; k0 < P.K; k0 += 8) {
+    const bool more = k0 + 8 < P.K;
+    if (more) gload(k0 + 8);
+#pragma unroll
+    for (int kk = 0; kk < 8; ++kk) {
+      const float4 a0 = *reinterpret_cast<const float4*>(&As[buf][kk][ty * 4]);
+      const float4 a1 = *reinterpret_cast<const float4*>(&As[buf][kk][64 + ty * 4]);
+      const float4 b0 = *reinterpret_cast<const float4*>(&Bs[buf][kk][tx * 4]);
+      const float4 b1 = *reinterpret_cast<const float4*>(&Bs[buf][kk][64 + tx * 4]);
+      const float a[8] = {a0.x, a0.y, a0.z, a0.w, a1.x, a1.y, a1.z, a1.w};
+      const float b[8] = {b0.x, b0.y, b0.z, b0.w, b1.x, b1.y, b1.z, b1.w};
+#pragma unroll
+      for (int i = 0; i < 8; ++i)
+#pragma unroll
+        for (int j = 0; j < 8; ++j) acc[i][j] = fmaf(a[i], b[j], acc[i][j]);
+    }
+    if (more) {
+      sstore(buf ^ 1);
+      __syncthreads();
+      buf ^= 1;
+    }
+  }
+#pragma unroll
+  for (int i = 0; i < 8; ++i) {
+    const int m = m0 + (i < 4 ? ty * 4 + i : 64 + ty * 4 + i - 4);
+    if (m >= P.M) continue;
+    float* crow = P.C + (int64_t)m * P.ldc;
+#pragma unroll
+    for (int h = 0; h < 2; ++h) {
+      const int n = n0 + h * 64 + tx * 4;
+      if (n + 3 < P.N) {
+        *reinterpret_cast<float4*>(crow + n) = make_float4(acc[i][4 * h], acc[i][4 * h + 1], acc[i][4 * h + 2], acc[i][4 * h + 3]);
+      } else {
+        for (int j = 0; j < 4; ++j)
+          if (n + j < P.N) crow[n + j] = acc[i][4 * h + j];
+      }
+    }
+  }
+}
+
 template <class V>
 __global__ void __launch_bounds__(256) t3_splitk_combine(const __grid_constant__ T3Params P) {
   const int64_t total = P.Z * P.M * P.N;
@@ -231,10 +329,52 @@ mdh_status prepare_t3(Plan* p) {
   p->tiles.split = S;
   p->tiles.bk = (int)std::min<int64_t>(kchunk, INT32_MAX);
   p->ws_kernel = S > 1 ? (size_t)S * c.Z * c.M * c.N * sizeof(float) : 0;
+  // linear fast path: fp32 A[m·lda + k], B[k·ldb + n], C[m·ldc + n], all 16-byte aligned
+  p->auxi.clear();
+  if (S == 1 && c.Z == 1 && p->in[c.a_buf].dtype == MDH_F32 && p->in[c.b_buf].dtype == MDH_F32 &&
+      p->out[0].dtype == MDH_F32 && c.M < INT32_MAX && c.N < INT32_MAX && c.K < INT32_MAX) {
+    const Access& A = p->in[c.a_buf].acc[0];
+    const Access& B = p->in[c.b_buf].acc[0];
+    const Access& C = p->out[0].acc[0];
+    auto lin = [&](const int* dims, int nd, const Access& acc, int64_t* s) {
+      std::vector<int64_t> t = group_table(*p, dims, nd, acc);
+      *s = t.size() > 1 ? t[1] - t[0] : 1;
+      for (size_t i = 1; i < t.size(); ++i)
+        if (t[i] - t[i - 1] != *s) return false;
+      return true;
+    };
+    int64_t sam, sak, sbk, sbn, scm, scn;
+    bool ok = lin(c.md, c.nm, A, &sam) && lin(c.kd, c.nk, A, &sak) && lin(c.kd, c.nk, B, &sbk) &&
+              lin(c.nd, c.nn, B, &sbn) && lin(c.md, c.nm, C, &scm) && lin(c.nd, c.nn, C, &scn);
+    if (c.K == 1) sak = 1;
+    if (c.N == 1) sbn = scn = 1;
+    if (c.M == 1) sam = scm = 4;
+    if (c.K == 1) sbk = 4;
+    ok = ok && sak == 1 && sbn == 1 && scn == 1 && sam % 4 == 0 && sbk % 4 == 0 && scm % 4 == 0 && A.base % 4 == 0 &&
+         B.base % 4 == 0 && C.base % 4 == 0 && sam < INT32_MAX && sbk < INT32_MAX && scm < INT32_MAX;
+    if (ok) p->auxi = {1, sam, sbk, scm, A.base, B.base, C.base};
+  }
   return MDH_OK;
 }
 
 mdh_status launch_t3(const Plan& p, const void* const* in, void* const* out, void* ws, cudaStream_t st) {
+  if (!p.auxi.empty() && p.auxi[0] == 1) {
+    const Contraction& c = p.con;
+    T3Lin L;
+    L.A = (const float*)in[c.a_buf] + p.auxi[4];
+    L.B = (const float*)in[c.b_buf] + p.auxi[5];
+    L.C = (float*)out[0] + p.auxi[6];
+    L.M = (int)c.M;
+    L.N = (int)c.N;
+    L.K = (int)c.K;
+    L.lda = (int)p.auxi[1];
+    L.ldb = (int)p.auxi[2];
+    L.ldc = (int)p.auxi[3];
+    dim3 grid((unsigned)((c.N + 127) / 128), (unsigned)((c.M + 127) / 128));
+    if (grid.y > 65535) { set_error("T3: grid too large"); return MDH_ERR_UNSUPPORTED; }
+    t3_linear_kernel<<<grid, 256, 0, st>>>(L);
+    return post_launch("t3_linear_kernel");
+  }
   const char* dc = nullptr;
   MDH_TRY(device_consts(p, &dc));
   const Contraction& c = p.con;

@@ -578,6 +578,23 @@ struct PermParams {
   int chunked;           // inner offsets contiguous in runs of 8 (aligned)
 };
 
+// chunked gather with a 2-D grid (blockIdx.y = outer row): no integer division per chunk,
+// two independent 16-byte chunks per thread in flight
+__global__ void __launch_bounds__(256) permute_rows_kernel(const __grid_constant__ PermParams P) {
+  const int64_t o = blockIdx.y;
+  const int64_t nc = P.nI / 8;
+  const uint16_t* src = P.src + P.offO[o];
+  uint16_t* dst = P.dst + o * P.ld;
+  for (int64_t c = (int64_t)blockIdx.x * 512 + threadIdx.x; c < nc; c += (int64_t)gridDim.x * 512) {
+    const int64_t c2 = c + 256;
+    const uint4 v0 = __ldg(reinterpret_cast<const uint4*>(src + __ldg(P.offI + c * 8)));
+    uint4 v1 = v0;
+    if (c2 < nc) v1 = __ldg(reinterpret_cast<const uint4*>(src + __ldg(P.offI + c2 * 8)));
+    *reinterpret_cast<uint4*>(dst + c * 8) = v0;
+    if (c2 < nc) *reinterpret_cast<uint4*>(dst + c2 * 8) = v1;
+  }
+}
+
 __global__ void __launch_bounds__(256) permute_kernel(const __grid_constant__ PermParams P) {
   if (P.chunked) {
     const int64_t nc = P.nI / 8;
@@ -889,6 +906,12 @@ static mdh_status run_permute(const t4::Layout2D& L, const uint16_t* src, char* 
   Q.chunked = L.chunked;
   if (L.mn_major) { Q.offO = offK; Q.offI = offMN; Q.nO = K; Q.nI = MN; }
   else { Q.offO = offMN; Q.offI = offK; Q.nO = MN; Q.nI = K; }
+  if (Q.chunked && Q.nO <= 65535) {
+    dim3 grid((unsigned)std::max<int64_t>(1, (Q.nI / 8 + 511) / 512), (unsigned)Q.nO);
+    t4::permute_rows_kernel<<<grid, 256, 0, st>>>(Q);
+    *out = Q.dst;
+    return post_launch("t4_permute_rows_kernel");
+  }
   const int64_t work = Q.chunked ? Q.nO * (Q.nI / 8) : Q.nO * Q.nI;
   const unsigned g = (unsigned)std::max<int64_t>(1, std::min<int64_t>((work + 255) / 256, 148LL * 32));
   t4::permute_kernel<<<g, 256, 0, st>>>(Q);
