@@ -90,6 +90,16 @@ def workload(name, world=1, rank=0):
         spec = S.mcc(256, 7, 7, 512, 3, 3, 512, "bf16")
         return dict(spec=spec, inputs=lambda: G.mcc_inputs(spec), work=2.0 * 256 * 49 * 512 * 4608, unit="TFLOP/s",
                     scale=1e12, bound="tensor", dtype="bf16", desc="MCC ResNet-50 conv5_1 3x3/s2 N=256 bf16")
+    if name == "prefix_sum_f32":
+        spec = S.prefix_sum([1 << 26], 0)
+        return dict(spec=spec, inputs=lambda: G.gen_inputs(spec, 6100, "positive"), work=8.0 * (1 << 26),
+                    unit="GB/s", scale=1e9, bound="hbm", dtype="f32",
+                    desc="ps(add) prefix sum of 2^26 fp32 (Listing 17; F1)")
+    if name == "mbbs_f32":
+        spec = S.mbbs(8192, 8192)
+        return dict(spec=spec, inputs=lambda: G.gen_inputs(spec, 6200, "positive"), work=4.0 * (8192 * 8192 + 8192),
+                    unit="GB/s", scale=1e9, bound="hbm", dtype="f32",
+                    desc="MBBS md_hom(id,(pw(add),ps(add))) over 8192^2 fp32 (F1)")
     if name in ("prl_A", "prl_B"):
         N, I = ((1 << 20), (1 << 14)) if name == "prl_A" else ((1 << 14), (1 << 20))
         spec = S.prl(N, I)
@@ -99,7 +109,7 @@ def workload(name, world=1, rank=0):
 
 
 SUITE = ["dot_f32", "dot_i32", "dot_f32_2^28", "matvec_f32", "jacobi3d", "matmul_f32", "matmul_bf16",
-         "ccsd_bf16", "mcc_bf16", "prl_A", "prl_B"]
+         "ccsd_bf16", "mcc_bf16", "prl_A", "prl_B", "prefix_sum_f32", "mbbs_f32"]
 
 
 def roofline(w, seconds, pk):

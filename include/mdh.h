@@ -77,10 +77,13 @@ typedef enum {
   MDH_PW_PRL_ARGMAX = 4,   /* custom pw over the PRL record: lexicographic max of      */
                            /* (id_measure==14, match_weight, match_id); associative and */
                            /* commutative (reading C-19)                                */
-  MDH_PW_PRL_PAPER = 5     /* custom pw, Listing 11 prl_max literally:     */
+  MDH_PW_PRL_PAPER = 5,    /* custom pw, Listing 11 prl_max literally:     */
                            /* res = lhs if lhs.id==14 && rhs.id!=14 else rhs;           */
                            /* associative, NOT commutative — order preserved (C-2)      */
-  /* MDH_PS_ADD: prefix-sum operator ps (Listing 17) — NEXT        */
+  MDH_PS_ADD = 6           /* ps(add): prefix sum (Listing 17): the dim is   */
+                           /* KEPT; result at index k = fold over [0, k] (inclusive),   */
+                           /* lhs = lower index range (reading C-25).  May be combined  */
+                           /* only with pw(add) dims (MBBS).            */
 } mdh_combine;
 
 /* Scalar functions SF ("arbitrary but pure"); a fixed catalog here. */

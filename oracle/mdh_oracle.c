@@ -51,7 +51,7 @@
 
 /* the oracle's own codes (independent of include/mdh.h) */
 enum { T_BF16 = 0, T_F32 = 1, T_F64 = 2, T_I32 = 3, T_U32 = 4, T_I64 = 5 };
-enum { C_CC = 0, C_ADD = 1, C_MAX = 2, C_MIN = 3, C_PRL_ARGMAX = 4, C_PRL_PAPER = 5 };
+enum { C_CC = 0, C_ADD = 1, C_MAX = 2, C_MIN = 3, C_PRL_ARGMAX = 4, C_PRL_PAPER = 5, C_PS_ADD = 6 };
 enum { S_MUL = 0, S_STENCIL = 1, S_PRL = 2, S_IDENTITY = 3 };
 enum { K_FLOAT = 0, K_I32 = 1, K_U32 = 2, K_I64 = 3, K_PRL = 4 };
 
@@ -118,7 +118,9 @@ static int decode(const int64_t* e, int64_t n, const double* fp, int nfp, ospec*
   s->nfp = nfp;
   for (int d = 0; d < s->D; ++d) {
     if (s->size[d] < 1) { seterr(err, cap, "size of dim %d < 1 (reading C-10)", d); return -1; }
-    if (s->op[d] == C_CC) s->cc[s->ncc++] = d; else s->red[s->nred++] = d;
+    /* cc and ps dims are kept in the result; pw and ps dims are folded */
+    if (s->op[d] == C_CC || s->op[d] == C_PS_ADD) s->cc[s->ncc++] = d;
+    if (s->op[d] != C_CC) s->red[s->nred++] = d;
   }
   return 0;
 }
@@ -132,7 +134,7 @@ static void coord_range(const ospec* s, const obuf* B, int a, int r, int is_out,
                         int64_t* lo, int64_t* hi) {
   int64_t l = B->off[a][r], h = B->off[a][r];
   for (int d = 0; d < s->D; ++d) {
-    int64_t ext = (is_out && s->op[d] != C_CC) ? 0 : s->size[d] - 1;
+    int64_t ext = (is_out && s->op[d] != C_CC && s->op[d] != C_PS_ADD) ? 0 : s->size[d] - 1;
     int64_t c = B->coeff[a][r][d];
     if (c > 0) h += c * ext; else l += c * ext;
   }
@@ -260,6 +262,7 @@ static void combine(const ospec* s, int op, const otuple* l, const otuple* r, ot
   int nc = (s->f == S_PRL) ? 3 : 1;
   switch (op) {
     case C_ADD:
+    case C_PS_ADD:
       for (int c = 0; c < nc; ++c) {
         if (s->kind == K_FLOAT) res->f[c] = l->f[c] + r->f[c];
         else res->i[c] = wrap(s->kind, (int64_t)((uint64_t)l->i[c] + (uint64_t)r->i[c]));
@@ -292,20 +295,24 @@ static void combine(const ospec* s, int op, const otuple* l, const otuple* r, ot
   }
 }
 
-/* FOLD(t, idx): reduce pw dims red[t..] */
-static void fold(const ospec* s, const void* const* in, int64_t* idx, int t, otuple* out) {
+/* FOLD(t, idx): reduce the non-cc dims red[t..].  A pw dim folds its
+ * whole range and collapses to index 0; a ps dim (prefix sum, Listing 17) keeps its index:
+ * the result at output index k is the fold over [0, k] (inclusive; for a contiguous split
+ * P|Q, res[q] = cf(lhs[max P], rhs[q]) with the lower index range as lhs, reading C-25). */
+static void fold(const ospec* s, const void* const* in, int64_t* idx, const int64_t* keep, int t, otuple* out) {
   if (t == s->nred) { leaf(s, in, idx, out); return; }
   int d = s->red[t];
+  int64_t last = s->op[d] == C_PS_ADD ? keep[d] : s->size[d] - 1;
   otuple acc, nxt, tmp;
   idx[d] = 0;
-  fold(s, in, idx, t + 1, &acc);
-  for (int64_t v = 1; v < s->size[d]; ++v) {
+  fold(s, in, idx, keep, t + 1, &acc);
+  for (int64_t v = 1; v <= last; ++v) {
     idx[d] = v;
-    fold(s, in, idx, t + 1, &nxt);
+    fold(s, in, idx, keep, t + 1, &nxt);
     combine(s, s->op[d], &acc, &nxt, &tmp);   /* lhs = lower index range */
     acc = tmp;
   }
-  idx[d] = 0;
+  idx[d] = s->op[d] == C_PS_ADD ? keep[d] : 0;   /* output index: ps kept, pw collapsed (C-4) */
   *out = acc;
 }
 
@@ -417,7 +424,9 @@ int mdho_eval(const int64_t* enc, int64_t n, const double* fp, int nfp,
       }
       if (s.ncc > 0) idx[s.cc[0]] = o;
       memset(&y, 0, sizeof(y));
-      fold(&s, in, idx, 0, &y);
+      int64_t keep[O_MAXD];
+      memcpy(keep, idx, sizeof(keep));
+      fold(&s, in, idx, keep, 0, &y);
       store(&s, out, idx, &y, mark, &collide);
     }
   }
@@ -450,7 +459,9 @@ int mdho_eval_points(const int64_t* enc, int64_t n, const double* fp, int nfp,
     memset(idx, 0, sizeof(idx));
     for (int t = 0; t < s.ncc; ++t) idx[s.cc[t]] = points[p * s.D + s.cc[t]];
     memset(&y, 0, sizeof(y));
-    fold(&s, in, idx, 0, &y);
+    int64_t keep[O_MAXD];
+    memcpy(keep, idx, sizeof(keep));
+    fold(&s, in, idx, keep, 0, &y);
     for (int b = 0; b < s.nout; ++b) {
       const obuf* B = &s.b[s.nin + b];
       int c = (s.f == S_PRL) ? b : 0;

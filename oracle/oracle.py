@@ -24,7 +24,7 @@ LIB = os.path.join(HERE, "libmdh_oracle.so")
 
 MAGIC = 0x4D44484F
 _DT = {"bf16": 0, "f32": 1, "f64": 2, "i32": 3, "u32": 4, "i64": 5}
-_OP = {"CC": 0, "PW_ADD": 1, "PW_MAX": 2, "PW_MIN": 3, "PW_PRL_ARGMAX": 4, "PW_PRL_PAPER": 5}
+_OP = {"CC": 0, "PW_ADD": 1, "PW_MAX": 2, "PW_MIN": 3, "PW_PRL_ARGMAX": 4, "PW_PRL_PAPER": 5, "PS_ADD": 6}
 _FN = {"MUL": 0, "STENCIL": 1, "PRL_COMPARE": 2, "IDENTITY": 3}
 _NP_IN = {"bf16": np.uint16, "f32": np.float32, "f64": np.float64, "i32": np.int32,
           "u32": np.uint32, "i64": np.int64}

@@ -117,6 +117,7 @@ static mdh_status run_template(const mdh::Plan& p, const void* const* in, void* 
     case T3_SIMT: return launch_t3(p, in, out, ws, st);
     case T4_TC: return launch_t4(p, in, out, ws, st);
     case T5_PRL: return launch_t5(p, in, out, ws, st);
+    case T6_SCAN: return launch_t6(p, in, out, ws, st);
   }
   set_error("unknown template");
   return MDH_ERR_INTERNAL;

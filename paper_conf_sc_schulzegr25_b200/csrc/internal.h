@@ -26,7 +26,8 @@ enum Template : int {
   T2_REDUCE = 2,    // streaming reduction (Dot, MatVec, row/column reductions)
   T3_SIMT = 3,      // fp32/int32 SIMT contraction (MatMul fp32, CCSD(T)/MCC fp32)
   T4_TC = 4,        // bf16 tcgen05 contraction (MatMul, CCSD(T), MCC)
-  T5_PRL = 5        // pairwise record linkage with custom ordered combine
+  T5_PRL = 5,       // pairwise record linkage with custom ordered combine
+  T6_SCAN = 6       // ps(add) prefix sums (Listing 17; MBBS)
 };
 
 const char* template_name(int t);
@@ -82,8 +83,9 @@ struct Plan {
   Buf out[MDH_MAX_BUFS];
   int n_in_acc = 0;                   // total input accesses
   // ---- classification ----
-  int ncc = 0, nred = 0;
-  int cc[MDH_MAX_D], red[MDH_MAX_D];
+  int ncc = 0, nred = 0, nps = 0;
+  int cc[MDH_MAX_D], red[MDH_MAX_D];  // cc: kept dims (cc and ps); red: folded dims (pw and ps)
+  int ps[MDH_MAX_D];                  // prefix-sum dims (Listing 17)
   mdh_combine redop = MDH_CC;         // the common pw operator (reading C-3), CC if none
   int64_t Ncc = 1, Nred = 1;
   mdh_dtype compute = MDH_F32;        // arithmetic type of f and ⊕
@@ -157,6 +159,8 @@ mdh_status launch_t4(const Plan& p, const void* const* in, void* const* out, voi
 bool t4_supported(const Plan& p, std::string* why);
 mdh_status prepare_t5(Plan* p);
 mdh_status launch_t5(const Plan& p, const void* const* in, void* const* out, void* ws, cudaStream_t st);
+mdh_status prepare_t6(Plan* p);
+mdh_status launch_t6(const Plan& p, const void* const* in, void* const* out, void* ws, cudaStream_t st);
 void release_t4(Plan* p);
 
 // ordered ⊗-fold of S partial output sets (K-combine)

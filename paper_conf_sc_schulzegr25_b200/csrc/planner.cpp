@@ -24,6 +24,7 @@ const char* template_name(int t) {
     case T3_SIMT: return "T3_simt_contraction";
     case T4_TC: return "T4_tcgen05_contraction";
     case T5_PRL: return "T5_prl_pairwise";
+    case T6_SCAN: return "T6_prefix_scan";
   }
   return "?";
 }
@@ -36,7 +37,8 @@ static void coord_range(const Plan& p, const mdh_index_fn& fn, int r, bool colla
                         int64_t* lo, int64_t* hi) {
   int64_t l = fn.offset[r], h = fn.offset[r];
   for (int d = 0; d < p.D; ++d) {
-    int64_t ext = (collapse_red && p.op[d] != MDH_CC) ? 0 : p.size[d] - 1;
+    // output index functions see pw indices = 0 (C-4); cc and ps indices are kept
+    int64_t ext = (collapse_red && p.op[d] != MDH_CC && p.op[d] != MDH_PS_ADD) ? 0 : p.size[d] - 1;
     int64_t c = fn.coeff[r][d];
     if (c > 0) h += c * ext; else l += c * ext;
   }
@@ -209,15 +211,15 @@ static mdh_status shard_rewrite(Plan* p) {
 static int choose_shard_dim(const Plan& p) {
   if (p.f == MDH_F_PRL_COMPARE && p.nred > 0) return p.red[0];   // §8(e): PRL shards the DB dim
   for (int t = 0; t < p.ncc; ++t)
-    if (p.size[p.cc[t]] >= p.world) return p.cc[t];
+    if (p.op[p.cc[t]] == MDH_CC && p.size[p.cc[t]] >= p.world) return p.cc[t];
   for (int t = 0; t < p.nred; ++t)
-    if (p.size[p.red[t]] >= p.world) return p.red[t];
+    if (p.op[p.red[t]] != MDH_PS_ADD && p.size[p.red[t]] >= p.world) return p.red[t];
   return -1;
 }
 
 // ---- contraction grouping (A0): M = dims only A uses, N = only B, batch = both -------
 static bool group_contraction(Plan* p) {
-  if (p->f != MDH_F_MUL || p->n_in != 2 || p->in[0].nacc != 1 || p->in[1].nacc != 1) return false;
+  if (p->nps > 0 || p->f != MDH_F_MUL || p->n_in != 2 || p->in[0].nacc != 1 || p->in[1].nacc != 1) return false;
   if (p->nred == 0 || p->redop != MDH_PW_ADD) return false;
   Contraction c;
   const Access& A = p->in[0].acc[0];
@@ -302,7 +304,10 @@ static mdh_status select_template(Plan* p) {
   // template choice (SURVEY §8(a) A0 decision table)
   p->tmpl = T0_GENERIC;
   p->why = "generic fallback";
-  if (p->f == MDH_F_PRL_COMPARE) {
+  if (p->nps > 0) {
+    p->tmpl = T6_SCAN;
+    p->why = "ps(add) dim: prefix-sum scan";
+  } else if (p->f == MDH_F_PRL_COMPARE) {
     p->tmpl = T5_PRL;
     p->why = "f = PRL_COMPARE";
   } else if (p->nred == 0) {
@@ -339,8 +344,8 @@ mdh_status build_plan(const mdh_spec* spec, const mdh_plan_opts* opts, Plan* p) 
       set_error("size of dim %d is %lld; sizes must be >= 1 (reading C-10)", d, (long long)spec->size[d]);
       return MDH_ERR_INVALID_SPEC;
     }
-    if ((int)spec->op[d] < MDH_CC || (int)spec->op[d] > MDH_PW_PRL_PAPER) {
-      set_error("dim %d: unknown combine operator %d (ps is not in this build)", d, (int)spec->op[d]);
+    if ((int)spec->op[d] < MDH_CC || (int)spec->op[d] > MDH_PS_ADD) {
+      set_error("dim %d: unknown combine operator %d", d, (int)spec->op[d]);
       return MDH_ERR_UNSUPPORTED;
     }
     p->size[d] = spec->size[d];
@@ -360,9 +365,15 @@ mdh_status build_plan(const mdh_spec* spec, const mdh_plan_opts* opts, Plan* p) 
   // classification
   p->ncc = p->nred = 0;
   p->redop = MDH_CC;
+  p->nps = 0;
   for (int d = 0; d < p->D; ++d) {
     if (p->op[d] == MDH_CC) p->cc[p->ncc++] = d;
-    else {
+    else if (p->op[d] == MDH_PS_ADD) {
+      // a ps dim is kept in the result (enumerated like cc) and folded over [0, k]
+      p->cc[p->ncc++] = d;
+      p->red[p->nred++] = d;
+      p->ps[p->nps++] = d;
+    } else {
       if (p->redop != MDH_CC && p->op[d] != p->redop) {
         set_error("dims use different pw operators; the result would depend on the split "
                   "(interchange law fails, reading C-3)");
@@ -371,6 +382,14 @@ mdh_status build_plan(const mdh_spec* spec, const mdh_plan_opts* opts, Plan* p) 
       p->redop = p->op[d];
       p->red[p->nred++] = d;
     }
+  }
+  if (p->nps > 0) {
+    if (p->redop != MDH_CC && p->redop != MDH_PW_ADD) {
+      set_error("ps(add) combines only with pw(add) dims (interchange law, reading C-3)");
+      return MDH_ERR_UNSUPPORTED;
+    }
+    if (spec->f == MDH_F_PRL_COMPARE) { set_error("ps with PRL_COMPARE is outside the catalog"); return MDH_ERR_UNSUPPORTED; }
+    p->redop = MDH_PW_ADD;
   }
   bool prl_op = p->redop == MDH_PW_PRL_ARGMAX || p->redop == MDH_PW_PRL_PAPER;
   if (prl_op != (p->f == MDH_F_PRL_COMPARE) && !(p->f == MDH_F_PRL_COMPARE && p->nred == 0)) {
@@ -426,6 +445,7 @@ mdh_status build_plan(const mdh_spec* spec, const mdh_plan_opts* opts, Plan* p) 
     int sd = opts->shard_dim >= 0 ? opts->shard_dim : choose_shard_dim(*p);
     if (sd < 0 || sd >= p->D) { set_error("no dimension can be sharded over %d ranks", p->world); return MDH_ERR_INVALID_ARG; }
     if (p->size[sd] < p->world) { set_error("shard dim %d has %lld < %d points", sd, (long long)p->size[sd], p->world); return MDH_ERR_INVALID_ARG; }
+    if (p->op[sd] == MDH_PS_ADD) { set_error("sharding a ps dim is not supported in this build"); return MDH_ERR_UNSUPPORTED; }
     p->shard_dim = sd;
     if (p->op[sd] != MDH_CC && !(p->flags & (MDH_PLAN_VIRTUAL_SHARD | MDH_PLAN_NO_COLLECTIVE)) && !p->comm) {
       set_error("a pw shard needs an NCCL communicator (mdh_comm_init) or MDH_PLAN_VIRTUAL_SHARD");
@@ -450,6 +470,7 @@ mdh_status build_plan(const mdh_spec* spec, const mdh_plan_opts* opts, Plan* p) 
     case T3_SIMT: MDH_TRY(prepare_t3(p)); break;
     case T4_TC: MDH_TRY(prepare_t4(p)); break;
     case T5_PRL: MDH_TRY(prepare_t5(p)); break;
+    case T6_SCAN: MDH_TRY(prepare_t6(p)); break;
   }
   // pw shard: room for the gathered partials of all ranks
   p->ws_comm = 0;

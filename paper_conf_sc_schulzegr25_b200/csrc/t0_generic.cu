@@ -12,7 +12,8 @@ namespace mdh {
 constexpr int T0_MAX_ACC = 24;
 
 struct T0Params {
-  int D, ncc, nred, op, f, nacc, nout;
+  int D, ncc, nred, op, f, nacc, nout, nps;
+  int kind[MDH_MAX_D];                // per dim: 0 cc, 1 pw, 2 ps (kept and folded over [0,k])
   int64_t size[MDH_MAX_D];
   int cc[MDH_MAX_D], red[MDH_MAX_D];
   int64_t Ncc, Nred;
@@ -35,17 +36,22 @@ __global__ void __launch_bounds__(128) t0_kernel(const __grid_constant__ T0Param
     for (int a = 0; a < P.nacc; ++a) off[a] = P.base[a];
     int64_t ooff = P.obase[0];
     int64_t rem = c;
+    int64_t lim[MDH_MAX_D];            // fold extent per dim: I_d (pw) or k+1 (ps)
+    for (int d = 0; d < P.D; ++d) lim[d] = P.size[d];
     for (int t = P.ncc - 1; t >= 0; --t) {
       int d = P.cc[t];
       int64_t v = rem % P.size[d];
       rem /= P.size[d];
-      for (int a = 0; a < P.nacc; ++a) off[a] += P.L[a][d] * v;
+      if (P.kind[d] == 2) lim[d] = v + 1;              // ps: inputs are folded from index 0
+      else for (int a = 0; a < P.nacc; ++a) off[a] += P.L[a][d] * v;
       ooff += P.oL[0][d] * v;
     }
     int64_t ridx[MDH_MAX_D];
     for (int t = 0; t < P.nred; ++t) ridx[t] = 0;
     V acc = (V)0;
-    for (int64_t r = 0; r < P.Nred; ++r) {
+    int64_t nred_here = 1;
+    for (int t = 0; t < P.nred; ++t) nred_here *= lim[P.red[t]];
+    for (int64_t r = 0; r < nred_here; ++r) {
       V y;
       if (P.f == MDH_F_STENCIL) {
         y = (V)P.w[0] * load_as<V>(P.ptr[0], P.dt[0], off[0]);
@@ -56,14 +62,14 @@ __global__ void __launch_bounds__(128) t0_kernel(const __grid_constant__ T0Param
         y = load_as<V>(P.ptr[0], P.dt[0], off[0]);
       }
       acc = (r == 0) ? y : combine_op<V>(P.op, acc, y);    // left fold, lhs = lower range
-      // odometer over the pw dims (last pw dim fastest = lexicographic order)
+      // odometer over the folded dims (last fastest = lexicographic order)
       for (int t = P.nred - 1; t >= 0; --t) {
         int d = P.red[t];
-        if (++ridx[t] < P.size[d]) {
+        if (++ridx[t] < lim[d]) {
           for (int a = 0; a < P.nacc; ++a) off[a] += P.L[a][d];
           break;
         }
-        for (int a = 0; a < P.nacc; ++a) off[a] -= P.L[a][d] * (P.size[d] - 1);
+        for (int a = 0; a < P.nacc; ++a) off[a] -= P.L[a][d] * (lim[d] - 1);
         ridx[t] = 0;
       }
     }
@@ -136,6 +142,9 @@ mdh_status launch_t0(const Plan& p, const void* const* in, void* const* out, voi
   P.D = p.D;
   P.ncc = p.ncc;
   P.nred = p.nred;
+  P.nps = p.nps;
+  for (int d = 0; d < MDH_MAX_D; ++d)
+    P.kind[d] = d >= p.D ? 0 : (p.op[d] == MDH_CC ? 0 : (p.op[d] == MDH_PS_ADD ? 2 : 1));
   P.op = p.redop;
   P.f = p.f;
   P.Ncc = p.Ncc;

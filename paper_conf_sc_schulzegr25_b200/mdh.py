@@ -23,7 +23,7 @@ LIB_PATH = os.path.join(HERE, "libmdh.so")
 
 DTYPE = {"bf16": 0, "f32": 1, "f64": 2, "i32": 3, "u32": 4, "i64": 5}
 DTYPE_NAME = {v: k for k, v in DTYPE.items()}
-OP = {"CC": 0, "PW_ADD": 1, "PW_MAX": 2, "PW_MIN": 3, "PW_PRL_ARGMAX": 4, "PW_PRL_PAPER": 5}
+OP = {"CC": 0, "PW_ADD": 1, "PW_MAX": 2, "PW_MIN": 3, "PW_PRL_ARGMAX": 4, "PW_PRL_PAPER": 5, "PS_ADD": 6}
 FN = {"MUL": 0, "STENCIL": 1, "PRL_COMPARE": 2, "IDENTITY": 3}
 STATUS = {0: "OK", 1: "INVALID_ARG", 2: "INVALID_SPEC", 3: "UNSUPPORTED", 4: "OUT_OF_MEMORY",
           5: "CUDA", 6: "NCCL", 7: "INTERNAL"}
