@@ -297,10 +297,17 @@ def main():
     import torch.distributed as dist
     from paper_conf_sc_schulzegr25_b200 import lib
     lib()
+    # MDH_BENCH_BACKEND=gloo and MDH_BENCH_SAME_GPU=1 exercise the N>1 launch on a
+    # single-GPU machine (every rank on cuda:0); the default is NCCL, one GPU per rank.
+    backend = os.environ.get("MDH_BENCH_BACKEND", "nccl")
+    local = 0 if os.environ.get("MDH_BENCH_SAME_GPU") == "1" else local
     torch.cuda.set_device(local)
     dev = torch.device("cuda", local)
     if world > 1:
-        dist.init_process_group("nccl", device_id=dev)
+        if backend == "nccl":
+            dist.init_process_group("nccl", device_id=dev)
+        else:
+            dist.init_process_group(backend)
     pk = peaks()
     l2 = torch.cuda.get_device_properties(dev).L2_cache_size
     flush = L2Flush(dev)
@@ -319,8 +326,8 @@ def main():
     t_total = sum(res["times"])
     et_total = sum(res["e2e_times"])
     if world > 1:
-        tt = torch.tensor([t_total, et_total], dtype=torch.float64, device=dev)
-        dist.all_reduce(tt, op=dist.ReduceOp.MAX)
+        tt = torch.tensor([t_total, et_total], dtype=torch.float64, device=dev if backend == "nccl" else "cpu")
+        dist.all_reduce(tt, op=dist.ReduceOp.MAX)          # max over ranks
         t_total, et_total = float(tt[0]), float(tt[1])
     w = res["w"]
     per_step = t_total / K

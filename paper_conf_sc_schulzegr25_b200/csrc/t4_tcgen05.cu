@@ -585,8 +585,9 @@ __global__ void __launch_bounds__(256) permute_rows_kernel(const __grid_constant
   const int64_t nc = P.nI / 8;
   const uint16_t* src = P.src + P.offO[o];
   uint16_t* dst = P.dst + o * P.ld;
-  for (int64_t c = (int64_t)blockIdx.x * 512 + threadIdx.x; c < nc; c += (int64_t)gridDim.x * 512) {
-    const int64_t c2 = c + 256;
+  const int64_t span = 2 * (int64_t)blockDim.x;
+  for (int64_t c = (int64_t)blockIdx.x * span + threadIdx.x; c < nc; c += (int64_t)gridDim.x * span) {
+    const int64_t c2 = c + blockDim.x;
     const uint4 v0 = __ldg(reinterpret_cast<const uint4*>(src + __ldg(P.offI + c * 8)));
     uint4 v1 = v0;
     if (c2 < nc) v1 = __ldg(reinterpret_cast<const uint4*>(src + __ldg(P.offI + c2 * 8)));
@@ -906,9 +907,12 @@ static mdh_status run_permute(const t4::Layout2D& L, const uint16_t* src, char* 
   Q.chunked = L.chunked;
   if (L.mn_major) { Q.offO = offK; Q.offI = offMN; Q.nO = K; Q.nI = MN; }
   else { Q.offO = offMN; Q.offI = offK; Q.nO = MN; Q.nI = K; }
-  if (Q.chunked && Q.nO <= 65535) {
-    dim3 grid((unsigned)std::max<int64_t>(1, (Q.nI / 8 + 511) / 512), (unsigned)Q.nO);
-    t4::permute_rows_kernel<<<grid, 256, 0, st>>>(Q);
+  if (Q.chunked && Q.nO <= 65535 && Q.nI / 8 >= 4096) {   // long rows only: measured slower on MCC rows (576 chunks)
+    // block sized to the row: ceil(nc/2) threads (multiple of 32, ≤ 256), two chunks each
+    const int64_t nc = Q.nI / 8;
+    const int tb = (int)std::min<int64_t>(256, std::max<int64_t>(32, ((nc + 1) / 2 + 31) / 32 * 32));
+    dim3 grid((unsigned)std::max<int64_t>(1, (nc + 2 * tb - 1) / (2 * tb)), (unsigned)Q.nO);
+    t4::permute_rows_kernel<<<grid, tb, 0, st>>>(Q);
     *out = Q.dst;
     return post_launch("t4_permute_rows_kernel");
   }

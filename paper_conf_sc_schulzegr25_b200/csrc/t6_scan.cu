@@ -41,10 +41,20 @@ struct T6Params {
   void* sums;     // V[Nc][nq]
 };
 
+// K1 with the pw range split over threadIdx.y (8 contiguous sub-ranges, folded in order
+// through shared memory): 32 consecutive (c, t) points per block row keep loads coalesced
 template <class V>
 __global__ void __launch_bounds__(256) t6_fold_kernel(const __grid_constant__ T6Params P) {
+  __shared__ V part[8][32];
   const int64_t total = P.Nc * P.T;
-  for (int64_t e = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; e < total; e += (int64_t)gridDim.x * blockDim.x) {
+  int64_t npts = 1;
+  for (int q = 0; q < P.npw; ++q) npts *= P.pwsize[q];
+  const int64_t per = (npts + 7) / 8;
+  for (int64_t eb = (int64_t)blockIdx.x * 32; eb < total; eb += (int64_t)gridDim.x * 32) {
+    const int64_t e = eb + threadIdx.x;
+    const int64_t r0 = min(npts, (int64_t)threadIdx.y * per), r1 = min(npts, r0 + per);
+    V acc = (V)0;
+    if (e < total && r0 < r1) {
     const int64_t c = e / P.T, t = e % P.T;
     int64_t off[2] = {P.base[0] + P.Lt[0] * t, P.base[1] + P.Lt[1] * t};
     int64_t rem = c;
@@ -54,14 +64,18 @@ __global__ void __launch_bounds__(256) t6_fold_kernel(const __grid_constant__ T6
       off[0] += P.Lrow[0][q] * v;
       off[1] += P.Lrow[1][q] * v;
     }
-    V acc = (V)0;
     int64_t idx[MDH_MAX_D];
-    int64_t npts = 1;
-    for (int q = 0; q < P.npw; ++q) { idx[q] = 0; npts *= P.pwsize[q]; }
-    for (int64_t r = 0; r < npts; ++r) {
+    int64_t rr = r0;
+    for (int q = P.npw - 1; q >= 0; --q) {      // odometer start = r0 (mixed radix)
+      idx[q] = rr % P.pwsize[q];
+      rr /= P.pwsize[q];
+      off[0] += P.Lpw[0][q] * idx[q];
+      off[1] += P.Lpw[1][q] * idx[q];
+    }
+    for (int64_t r = r0; r < r1; ++r) {
       const V x0 = load_as<V>(P.ptr[0], P.dt[0], off[0]);
       const V y = (P.f == MDH_F_MUL) ? Arith<V>::mul(x0, load_as<V>(P.ptr[1], P.dt[1], off[1])) : x0;
-      acc = (r == 0) ? y : Arith<V>::add(acc, y);
+      acc = (r == r0) ? y : Arith<V>::add(acc, y);
       for (int q = P.npw - 1; q >= 0; --q) {
         if (++idx[q] < P.pwsize[q]) { off[0] += P.Lpw[0][q]; off[1] += P.Lpw[1][q]; break; }
         off[0] -= P.Lpw[0][q] * (P.pwsize[q] - 1);
@@ -69,7 +83,15 @@ __global__ void __launch_bounds__(256) t6_fold_kernel(const __grid_constant__ T6
         idx[q] = 0;
       }
     }
-    ((V*)P.z)[e] = acc;
+    }
+    part[threadIdx.y][threadIdx.x] = acc;
+    __syncthreads();
+    if (threadIdx.y == 0 && e < total) {
+      V s = part[0][threadIdx.x];
+      for (int y = 1; y < 8; ++y) s = Arith<V>::add(s, part[y][threadIdx.x]);   // sub-range order
+      ((V*)P.z)[e] = s;
+    }
+    __syncthreads();
   }
 }
 
@@ -88,8 +110,10 @@ __device__ __forceinline__ int64_t t6_out_offset(const T6Params& P, int64_t c, i
 template <class V>
 __global__ void __launch_bounds__(T6_THREADS) t6_chunk_scan_kernel(const __grid_constant__ T6Params P) {
   __shared__ V wsum[T6_THREADS / 32];
+  __shared__ V tile[T6_CHUNK + T6_CHUNK / 32];      // padded: thread k reads 16 consecutive
   const int64_t c = blockIdx.y, q = blockIdx.x;
-  const int64_t t0 = q * T6_CHUNK + (int64_t)threadIdx.x * T6_PER;
+  const int64_t tb = q * T6_CHUNK;
+  const int64_t t0 = tb + (int64_t)threadIdx.x * T6_PER;
   const V* zr = (const V*)P.z + c * P.T;
   // no pw dims and f = IDENTITY: scan the input directly (K1 skipped)
   int64_t xrow = P.base[0];
@@ -101,12 +125,20 @@ __global__ void __launch_bounds__(T6_THREADS) t6_chunk_scan_kernel(const __grid_
       xrow += P.Lrow[0][d] * v;
     }
   }
+  // coalesced staging of the chunk (consecutive threads, consecutive elements)
+#pragma unroll
+  for (int k = 0; k < T6_PER; ++k) {
+    const int j = k * T6_THREADS + threadIdx.x;
+    const int64_t t = tb + j;
+    tile[j + (j >> 5)] = t < P.T ? (P.direct ? load_as<V>(P.ptr[0], P.dt[0], xrow + P.Lt[0] * t) : zr[t]) : (V)0;
+  }
+  __syncthreads();
   V v[T6_PER];
   V run = (V)0;
 #pragma unroll
   for (int k = 0; k < T6_PER; ++k) {
-    const int64_t t = t0 + k;
-    const V x = t < P.T ? (P.direct ? load_as<V>(P.ptr[0], P.dt[0], xrow + P.Lt[0] * t) : zr[t]) : (V)0;
+    const int j = threadIdx.x * T6_PER + k;
+    const V x = tile[j + (j >> 5)];
     run = k == 0 ? x : Arith<V>::add(run, x);
     v[k] = run;
   }
@@ -125,27 +157,55 @@ __global__ void __launch_bounds__(T6_THREADS) t6_chunk_scan_kernel(const __grid_
   const V prev = __shfl_up_sync(0xffffffffu, incl, 1);     // inclusive total of lane-1
   const V excl = lane == 0 ? base : Arith<V>::add(base, prev);
   const bool single = P.nq == 1;
+  __syncthreads();
 #pragma unroll
   for (int k = 0; k < T6_PER; ++k) {
-    const int64_t t = t0 + k;
+    const int j = threadIdx.x * T6_PER + k;
+    tile[j + (j >> 5)] = (threadIdx.x == 0 && warp == 0) ? v[k] : Arith<V>::add(excl, v[k]);
+  }
+  __syncthreads();
+  // coalesced write-back
+#pragma unroll
+  for (int k = 0; k < T6_PER; ++k) {
+    const int j = k * T6_THREADS + threadIdx.x;
+    const int64_t t = tb + j;
     if (t >= P.T) break;
-    const V r = (threadIdx.x == 0 && warp == 0) ? v[k] : Arith<V>::add(excl, v[k]);
+    const V r = tile[j + (j >> 5)];
     if (single) store_as<V>(P.out, P.odt, t6_out_offset(P, c, t), r);
     else ((V*)P.loc)[c * P.T + t] = r;
   }
   if (!single && threadIdx.x == T6_THREADS - 1) ((V*)P.sums)[c * P.nq + q] = Arith<V>::add(excl, run);
 }
 
+// exclusive scan of each row's chunk totals, in chunk order: one CTA per row, tiles of
+// 256 totals scanned with warp shuffles and a running carry (fixed association order)
 template <class V>
 __global__ void __launch_bounds__(256) t6_sums_kernel(const __grid_constant__ T6Params P) {
-  // exclusive scan of the chunk totals of each row, in chunk order (one thread per row)
-  for (int64_t c = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; c < P.Nc; c += (int64_t)gridDim.x * blockDim.x) {
+  __shared__ V wsum[8];
+  const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+  for (int64_t c = blockIdx.x; c < P.Nc; c += gridDim.x) {
     V* s = (V*)P.sums + c * P.nq;
-    V acc = (V)0;
-    for (int64_t q = 0; q < P.nq; ++q) {
-      const V x = s[q];
-      s[q] = acc;
-      acc = q == 0 ? x : Arith<V>::add(acc, x);
+    V carry = (V)0;
+    for (int64_t q0 = 0; q0 < P.nq; q0 += 256) {
+      const int64_t q = q0 + threadIdx.x;
+      const V x = q < P.nq ? s[q] : (V)0;
+      V incl = x;
+#pragma unroll
+      for (int o = 1; o < 32; o <<= 1) {
+        const V n = __shfl_up_sync(0xffffffffu, incl, o);
+        if (lane >= o) incl = Arith<V>::add(n, incl);
+      }
+      __syncthreads();
+      if (lane == 31) wsum[warp] = incl;
+      __syncthreads();
+      V base = carry;
+      for (int w = 0; w < warp; ++w) base = Arith<V>::add(base, wsum[w]);
+      const V prev = __shfl_up_sync(0xffffffffu, incl, 1);
+      const V excl = lane == 0 ? base : Arith<V>::add(base, prev);
+      if (q < P.nq) s[q] = excl;
+      V tot = carry;
+      for (int w = 0; w < 8; ++w) tot = Arith<V>::add(tot, wsum[w]);
+      carry = tot;
     }
   }
 }
@@ -188,7 +248,8 @@ static mdh_status launch_typed(const T6Params& P, cudaStream_t st) {
   const int64_t total = P.Nc * P.T;
   const unsigned g = (unsigned)std::max<int64_t>(1, std::min<int64_t>((total + 255) / 256, 148LL * 32));
   if (!P.direct) {
-    t6_fold_kernel<V><<<g, 256, 0, st>>>(P);
+    const unsigned gf = (unsigned)std::max<int64_t>(1, std::min<int64_t>((total + 31) / 32, 148LL * 64));
+    t6_fold_kernel<V><<<gf, dim3(32, 8), 0, st>>>(P);
     MDH_TRY(post_launch("t6_fold_kernel"));
   }
   if (P.Nc > 65535) { set_error("T6: too many rows"); return MDH_ERR_UNSUPPORTED; }
@@ -196,7 +257,7 @@ static mdh_status launch_typed(const T6Params& P, cudaStream_t st) {
   t6_chunk_scan_kernel<V><<<grid, T6_THREADS, 0, st>>>(P);
   MDH_TRY(post_launch("t6_chunk_scan_kernel"));
   if (P.nq > 1) {
-    t6_sums_kernel<V><<<(unsigned)std::max<int64_t>(1, (P.Nc + 255) / 256), 256, 0, st>>>(P);
+    t6_sums_kernel<V><<<(unsigned)std::min<int64_t>(P.Nc, 148LL * 8), 256, 0, st>>>(P);
     MDH_TRY(post_launch("t6_sums_kernel"));
     t6_fix_kernel<V><<<g, 256, 0, st>>>(P);
     MDH_TRY(post_launch("t6_fix_kernel"));
