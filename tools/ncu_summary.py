@@ -68,7 +68,7 @@ def main():
     traffic_path = os.path.join(ROOT, "profiles", "ncu_traffic.json")
     traffic = json.load(open(traffic_path)) if os.path.exists(traffic_path) else {}
     for rep in a.reps:
-        wl = os.path.basename(rep).replace("prof_", "").replace(".ncu-rep", "")
+        wl = os.path.basename(rep).replace(".ncu-rep", "").split("_", 1)[1]
         for d in raw(rep):
             f = lambda k, s=1.0, p=1: (f"{d[k] / s:.{p}f}" if isinstance(d.get(k), float) else str(d.get(k, "")))
             lines.append(f"| {wl} | `{d['kernel'][:60]}` | {f('duration', 1e-6)} | {f('dram_read', 1e6)} | "
