@@ -66,7 +66,25 @@ struct Params {
   const int64_t* cM;                // generic output tables
   const int64_t* cN;
   int sched;                        // 0: round-robin, M-major; 1: contiguous range per CTA, N-major
+  // 2-SM split-K tail: units [0, nfull) are whole tiles; the remaining tiles are split into
+  // ssplit contiguous k-ranges each (units nfull + i·ssplit + s) whose fp32 partial tiles go
+  // to `part` and are folded in split order by tail_combine_kernel
+  int nunits, nfull, ssplit;
+  float* part;
+  unsigned* tail_cnt;               // 2 counters per split tile (arrivals, departures); zero at rest
 };
+
+__device__ __forceinline__ void unit_decode(const Params& P, int u, int* t, int* kb0, int* kb1, int* slot) {
+  if (u < P.nfull) {
+    *t = u; *kb0 = 0; *kb1 = P.num_kb; *slot = -1;
+  } else {
+    const int v = u - P.nfull, i = v / P.ssplit, s = v % P.ssplit;
+    *t = P.nfull + i;
+    *kb0 = (int)((int64_t)s * P.num_kb / P.ssplit);
+    *kb1 = (int)((int64_t)(s + 1) * P.num_kb / P.ssplit);
+    *slot = v;
+  }
+}
 
 // Tile schedule shared by the three roles.  Round-robin M-major keeps concurrently running
 // CTAs on neighbouring tiles (operand reuse in L2); the contiguous N-major range keeps one
@@ -453,6 +471,7 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(THREADS, 1)
   }
   tc_fence_before();
   cluster_sync_all();
+  __syncthreads();               // (also orders the TMEM-address slot for racecheck)
   tc_fence_after();
   const uint32_t tmem = *tmem_slot;
 
@@ -461,9 +480,11 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(THREADS, 1)
       // ===== TMA producer (both CTAs; bytes are counted at the leader's full barrier) =====
       int stage = 0;
       uint32_t phase = 0;
-      for (int t = cluster_id; t < P.num_tiles; t += nclusters) {
+      for (int u = cluster_id; u < P.nunits; u += nclusters) {
+        int t, kb0, kb1, slot;
+        unit_decode(P, u, &t, &kb0, &kb1, &slot);
         const int m0 = (t / P.tiles_n) * 256 + (int)rank * 128, n0 = (t % P.tiles_n) * 256 + (int)rank * 128;
-        for (int kb = 0; kb < P.num_kb; ++kb) {
+        for (int kb = kb0; kb < kb1; ++kb) {
           mbar_wait(empty0 + 8 * stage, phase ^ 1);
           const uint32_t fb_leader = map_to_rank0(full0 + 8 * stage);
           if (leader) mbar_expect_tx(full0 + 8 * stage, 2 * STAGE2_BYTES);
@@ -492,12 +513,14 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(THREADS, 1)
       int stage = 0;
       uint32_t phase = 0;
       int it = 0;
-      for (int t = cluster_id; t < P.num_tiles; t += nclusters, ++it) {
+      for (int u = cluster_id; u < P.nunits; u += nclusters, ++it) {
+        int t, kb0, kb1, slot;
+        unit_decode(P, u, &t, &kb0, &kb1, &slot);
         const int acc = it & 1;
         mbar_wait(tempty0 + 8 * acc, ((it >> 1) & 1) ^ 1);
         tc_fence_after();
         const uint32_t d = tmem + acc * BN;
-        for (int kb = 0; kb < P.num_kb; ++kb) {
+        for (int kb = kb0; kb < kb1; ++kb) {
           mbar_wait(full0 + 8 * stage, phase);
           tc_fence_after();
           const uint32_t a0 = smem_u32(sA + stage * A2_BYTES), b0 = smem_u32(sB + stage * B2_BYTES);
@@ -505,7 +528,7 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(THREADS, 1)
           for (int k = 0; k < BK / 16; ++k) {
             const uint64_t ad = P.a_mn_major ? sdesc(a0 + 2048 * k, 8192, 1024) : sdesc(a0 + 32 * k, 16, 1024);
             const uint64_t bd = P.b_mn_major ? sdesc(b0 + 2048 * k, 8192, 1024) : sdesc(b0 + 32 * k, 16, 1024);
-            mma_bf16_cg2(d, ad, bd, P.idesc, (kb | k) != 0);
+            mma_bf16_cg2(d, ad, bd, P.idesc, (kb != kb0) || k != 0);
           }
           mma_commit_cg2(empty0 + 8 * stage);
           if (++stage == S2) { stage = 0; phase ^= 1; }
@@ -525,7 +548,9 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(THREADS, 1)
     const int row = quad * 32 + lane;
     const uint32_t tempty_leader = map_to_rank0(tempty0);
     int it = 0;
-    for (int t = cluster_id; t < P.num_tiles; t += nclusters, ++it) {
+    for (int u = cluster_id; u < P.nunits; u += nclusters, ++it) {
+      int t, kb0, kb1, slot;
+      unit_decode(P, u, &t, &kb0, &kb1, &slot);
       const int acc = it & 1;
       const int64_t m = (int64_t)(t / P.tiles_n) * 256 + rank * 128 + row;
       const int64_t n0 = (int64_t)(t % P.tiles_n) * 256 + half * 128;
@@ -533,12 +558,49 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(THREADS, 1)
       tc_fence_after();
       const bool mok = m < P.M;
       const int64_t crow = P.cbase + (OUT_ROWMAJOR ? (mok ? m : 0) * P.ldc : __ldg(P.cM + (mok ? m : 0)));
+      // split-K tail: splits 0..S-2 write a dense fp32 partial tile [256][256] (row =
+      // rank·128 + row) to the workspace and count themselves in at the tile's counter; the
+      // last split (all split units run in the same, final wave) waits for them and folds
+      // p_0 + p_1 + … + own in split order before writing the output
+      const bool split = slot >= 0;
+      const int sidx = split ? slot % P.ssplit : 0, ti = split ? slot / P.ssplit : 0;
+      const bool last = split && sidx == P.ssplit - 1;
+      unsigned* cnt = P.tail_cnt + 2 * ti;
+      const int64_t prel = (int64_t)(rank * 128 + row) * 256 + half * 128;
+      float* prow = (split && !last) ? P.part + (int64_t)slot * 65536 + prel : nullptr;
+      if (last) {
+        if (lane == 0)
+          while (*((volatile unsigned*)cnt) < 16u * (unsigned)(P.ssplit - 1)) __nanosleep(64);
+        __syncwarp();
+        __threadfence();
+      }
 #pragma unroll 1
       for (int c = 0; c < 4; ++c) {
         uint32_t r[32];
         tmem_ld32(tmem + ((uint32_t)(quad * 32) << 16) + acc * BN + half * 128 + c * 32, r);
         const int64_t nb = n0 + c * 32;
-        if (OUT_ROWMAJOR && mok && nb + 32 <= P.N && ((crow + nb) & 3) == 0) {
+        if (last) {
+          const float* p0 = P.part + (int64_t)(ti * P.ssplit) * 65536 + prel + c * 32;
+#pragma unroll
+          for (int j4 = 0; j4 < 8; ++j4) {
+            float4 a = *reinterpret_cast<const float4*>(p0 + 4 * j4);
+            for (int s2 = 1; s2 < P.ssplit - 1; ++s2) {
+              const float4 b = *reinterpret_cast<const float4*>(p0 + (int64_t)s2 * 65536 + 4 * j4);
+              a.x += b.x; a.y += b.y; a.z += b.z; a.w += b.w;
+            }
+            r[4 * j4] = __float_as_uint(a.x + __uint_as_float(r[4 * j4]));
+            r[4 * j4 + 1] = __float_as_uint(a.y + __uint_as_float(r[4 * j4 + 1]));
+            r[4 * j4 + 2] = __float_as_uint(a.z + __uint_as_float(r[4 * j4 + 2]));
+            r[4 * j4 + 3] = __float_as_uint(a.w + __uint_as_float(r[4 * j4 + 3]));
+          }
+        }
+        if (prow) {
+          float4* dst = reinterpret_cast<float4*>(prow + c * 32);
+#pragma unroll
+          for (int j = 0; j < 8; ++j)
+            dst[j] = make_float4(__uint_as_float(r[4 * j]), __uint_as_float(r[4 * j + 1]), __uint_as_float(r[4 * j + 2]),
+                                 __uint_as_float(r[4 * j + 3]));
+        } else if (OUT_ROWMAJOR && mok && nb + 32 <= P.N && ((crow + nb) & 3) == 0) {
           float4* dst = reinterpret_cast<float4*>(P.C + crow + nb);
 #pragma unroll
           for (int j = 0; j < 8; ++j)
@@ -548,6 +610,17 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(THREADS, 1)
 #pragma unroll
           for (int j = 0; j < 32; ++j)
             if (nb + j < P.N) P.C[crow + (OUT_ROWMAJOR ? nb + j : __ldg(P.cN + nb + j))] = __uint_as_float(r[j]);
+        }
+      }
+      if (split && !last) {            // publish this warp's part of the partial tile
+        __threadfence();
+        __syncwarp();
+        if (lane == 0) atomicAdd(cnt, 1u);
+      } else if (last) {               // 16 warps (2 CTAs × 8) leave; the last one resets
+        __syncwarp();
+        if (lane == 0 && atomicAdd(cnt + 1, 1u) == 15u) {
+          cnt[0] = 0u;
+          cnt[1] = 0u;
         }
       }
       tc_fence_before();
@@ -563,6 +636,25 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(THREADS, 1)
     asm volatile("tcgen05.dealloc.cta_group::2.sync.aligned.b32 %0, %1;" ::"r"(tmem), "r"(TMEM_COLS));
   }
 }
+
+// fold the split-K partial tiles of the tail in split order and write them through out_view
+__global__ void __launch_bounds__(256) tail_combine_kernel(const __grid_constant__ Params P) {
+  const int ntail = (P.nunits - P.nfull) / P.ssplit;
+  const int64_t total = (int64_t)ntail * 65536;
+  for (int64_t e = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; e < total; e += (int64_t)gridDim.x * blockDim.x) {
+    const int i = (int)(e >> 16), rc = (int)(e & 65535), r = rc >> 8, c = rc & 255;
+    const int t = P.nfull + i;
+    const int64_t m = (int64_t)(t / P.tiles_n) * 256 + r, n = (int64_t)(t % P.tiles_n) * 256 + c;
+    if (m >= P.M || n >= P.N) continue;
+    const float* src = P.part + (int64_t)i * P.ssplit * 65536 + rc;
+    float acc = src[0];
+    for (int s = 1; s < P.ssplit; ++s) acc += src[(int64_t)s * 65536];
+    const int64_t o = P.cbase + (P.c_rowmajor ? m * P.ldc + n : P.cM[m] + P.cN[n]);
+    P.C[o] = acc;
+  }
+}
+
+constexpr int MAX_TAIL_UNITS = 74;   // partial tiles reserved in the workspace (2-SM path)
 
 // ---- operand normalisation pre-pass ---------------------------------------------------
 // An operand whose (MN, K) offsets are not 2-D linear (e.g. CCSD(T)'s t2 in output order,
@@ -593,6 +685,28 @@ __global__ void __launch_bounds__(256) permute_rows_kernel(const __grid_constant
     if (c2 < nc) v1 = __ldg(reinterpret_cast<const uint4*>(src + __ldg(P.offI + c2 * 8)));
     *reinterpret_cast<uint4*>(dst + c * 8) = v0;
     if (c2 < nc) *reinterpret_cast<uint4*>(dst + c2 * 8) = v1;
+  }
+}
+
+// chunked gather, one warp per outer row: 32-bit chunk indices, 4 independent 16-byte loads
+// in flight per lane, coalesced stores along the row
+__global__ void __launch_bounds__(256) permute_warp_kernel(const __grid_constant__ PermParams P) {
+  const int lane = threadIdx.x & 31;
+  const int nc = (int)(P.nI / 8);
+  const int64_t warps = (int64_t)gridDim.x * (blockDim.x >> 5);
+  for (int64_t o = blockIdx.x * (int64_t)(blockDim.x >> 5) + (threadIdx.x >> 5); o < P.nO; o += warps) {
+    const uint16_t* src = P.src + P.offO[o];
+    uint16_t* dst = P.dst + o * P.ld;
+    int c = lane;
+    for (; c + 96 < nc; c += 128) {
+      uint4 v[4];
+#pragma unroll
+      for (int u = 0; u < 4; ++u) v[u] = __ldg(reinterpret_cast<const uint4*>(src + __ldg(P.offI + (int64_t)(c + 32 * u) * 8)));
+#pragma unroll
+      for (int u = 0; u < 4; ++u) *reinterpret_cast<uint4*>(dst + (int64_t)(c + 32 * u) * 8) = v[u];
+    }
+    for (; c < nc; c += 32)
+      *reinterpret_cast<uint4*>(dst + (int64_t)c * 8) = __ldg(reinterpret_cast<const uint4*>(src + __ldg(P.offI + (int64_t)c * 8)));
   }
 }
 
@@ -723,6 +837,7 @@ struct T4State {
   t4::Layout2D a, b;
   t4::Params P;
   int cg = 1;      // 1: one SM per 128×256 tile; 2: SM pair per 256×256 tile
+  size_t tail_off = 0;
   // implicit-GEMM A map (a_box): TMA-order dims, byte strides, box
   int brank = 0;
   uint64_t bdims[5], bstrides[4];
@@ -850,6 +965,10 @@ mdh_status prepare_t4(Plan* p) {
     P.tiles_n = (int)((c.N + 255) / 256);
     P.num_tiles = P.tiles_m * P.tiles_n;
     P.idesc = (P.idesc & ~(0x1Fu << 24)) | ((uint32_t)(256 >> 4) << 24);
+    // room for the split-K tail's partial tiles (decided at launch from the SM count)
+    ws = (ws + 255) / 256 * 256;
+    s->tail_off = ws;
+    ws += (size_t)t4::MAX_TAIL_UNITS * 65536 * sizeof(float) + 2 * t4::MAX_TAIL_UNITS * sizeof(unsigned) + 256;
   }
   p->tmaps = s;
   p->t4_variant = 1 + (s->a.permuted ? 2 : 0) + (s->b.permuted ? 4 : 0) + (s->cg == 2 ? 8 : 0) + (a_box ? 16 : 0);
@@ -907,6 +1026,12 @@ static mdh_status run_permute(const t4::Layout2D& L, const uint16_t* src, char* 
   Q.chunked = L.chunked;
   if (L.mn_major) { Q.offO = offK; Q.offI = offMN; Q.nO = K; Q.nI = MN; }
   else { Q.offO = offMN; Q.offI = offK; Q.nO = MN; Q.nI = K; }
+  if (Q.chunked && Q.nI / 8 >= 32 && Q.nI / 8 < INT32_MAX) {
+    const unsigned g = (unsigned)std::max<int64_t>(1, std::min<int64_t>((Q.nO + 7) / 8, 148LL * 16));
+    t4::permute_warp_kernel<<<g, 256, 0, st>>>(Q);
+    *out = Q.dst;
+    return post_launch("t4_permute_warp_kernel");
+  }
   if (Q.chunked && Q.nO <= 65535 && Q.nI / 8 >= 4096) {   // long rows only: measured slower on MCC rows (576 chunks)
     // block sized to the row: ceil(nc/2) threads (multiple of 32, ≤ 256), two chunks each
     const int64_t nc = Q.nI / 8;
@@ -980,7 +1105,26 @@ mdh_status launch_t4(const Plan& p, const void* const* in, void* const* out, voi
   cudaGetDevice(&dev);
   cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
   if (s->cg == 2) {
-    const int grid2 = 2 * std::min(P.num_tiles, sms / 2);
+    // optional split-K tail (tile knob split=S ≥ 2): whole tiles for the complete waves, the
+    // last partial wave's tiles split along K over the idle SM pairs.  Off by default: on
+    // MatMul 4096³ and MCC conv5_1 it measured slower than whole tiles.
+    const int C = std::max(1, std::min(P.num_tiles, sms / 2));
+    const int T = P.num_tiles, R = T / C, Tr = T - R * C;
+    int S = 1;
+    if (Tr > 0 && p.tiles.split > 1) S = std::min({p.tiles.split, C / Tr, t4::MAX_TAIL_UNITS / Tr, P.num_kb});
+    if (S >= 2) {
+      P.nfull = T - Tr;
+      P.ssplit = S;
+      P.nunits = P.nfull + Tr * S;
+      P.part = (float*)((char*)ws + s->tail_off);
+      P.tail_cnt = (unsigned*)((char*)ws + s->tail_off + (size_t)t4::MAX_TAIL_UNITS * 65536 * sizeof(float));
+    } else {
+      P.nfull = T;
+      P.ssplit = 1;
+      P.nunits = T;
+      P.part = nullptr;
+    }
+    const int grid2 = 2 * std::max(1, std::min(P.nunits, sms / 2));
     t4::gemm2_kernel<true><<<grid2, t4::THREADS, t4::SMEM2_BYTES, st>>>(ma, mb, P);
     return post_launch("t4_gemm2_kernel");
   }
