@@ -67,7 +67,8 @@ struct Tiles {
   int zchunk = 32;
   int per_thread = 1;
   int cluster = 1;
-  int implicit = 0;                   // T4: implicit-GEMM (N-d TMA box) A operand instead of a gather
+  int implicit = 0;                   // T4 A operand when not 2-D: 0 auto, 1 N-d TMA box (implicit
+                                      // GEMM), 2 in-kernel cp.async gather, 3 gather pre-pass
   std::string source = "default";
 };
 

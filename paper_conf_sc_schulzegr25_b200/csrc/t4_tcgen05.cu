@@ -72,7 +72,24 @@ struct Params {
   int nunits, nfull, ssplit;
   float* part;
   unsigned* tail_cnt;               // 2 counters per split tile (arrivals, departures); zero at rest
+  // gather producer for A (AG kernels): A[m, k] = Ag[aM[m] + akoff[k/8] + k%8], K % 8 == 0
+  const uint16_t* Ag;
+  const int64_t* aM;
+  const int64_t* aK;                // offA_K table (every 8th entry is a chunk start)
+  int nkc;                          // K / 8 chunk offsets staged in shared memory
+  int ag_lag;                       // k-blocks between issuing a stage and publishing it (1..3)
 };
+
+constexpr int AG_WARPS = 4, AG_THREADS = AG_WARPS * 32, KOFF_MAX = 2048;
+constexpr int SMEM_AG_BYTES = STAGES * STAGE_BYTES + 1024 + 256 + KOFF_MAX * 8;
+
+__device__ __forceinline__ void cp_async16(uint32_t dst, const void* src) {
+  asm volatile("cp.async.cg.shared.global [%0], [%1], 16;" ::"r"(dst), "l"(src) : "memory");
+}
+__device__ __forceinline__ void cp_async_commit() { asm volatile("cp.async.commit_group;" ::: "memory"); }
+template <int N>
+__device__ __forceinline__ void cp_async_wait() { asm volatile("cp.async.wait_group %0;" ::"n"(N) : "memory"); }
+__device__ __forceinline__ void fence_proxy_async() { asm volatile("fence.proxy.async.shared::cta;" ::: "memory"); }
 
 __device__ __forceinline__ void unit_decode(const Params& P, int u, int* t, int* kb0, int* kb1, int* slot) {
   if (u < P.nfull) {
@@ -100,6 +117,17 @@ __device__ __forceinline__ int t_step(const Params& P) { return P.sched ? 1 : (i
 __device__ __forceinline__ void t_decode(const Params& P, int t, int* mb, int* nb) {
   if (P.sched) { *nb = t / P.tiles_m; *mb = t % P.tiles_m; }
   else { *mb = t / P.tiles_n; *nb = t % P.tiles_n; }
+}
+// 1-SM work units: whole tiles (ssplit ≤ 1, schedule above), or with a split-K tail the
+// units of unit_decode, round-robin (host sets sched = 0)
+__device__ __forceinline__ int u_first(const Params& P) { return P.ssplit > 1 ? (int)blockIdx.x : t_first(P); }
+__device__ __forceinline__ int u_last(const Params& P) { return P.ssplit > 1 ? P.nunits : t_last(P); }
+__device__ __forceinline__ int u_step(const Params& P) { return P.ssplit > 1 ? (int)gridDim.x : t_step(P); }
+__device__ __forceinline__ void u_decode(const Params& P, int u, int* mb, int* nb, int* kb0, int* kb1, int* slot) {
+  int t = u;
+  if (P.ssplit > 1) unit_decode(P, u, &t, kb0, kb1, slot);
+  else { *kb0 = 0; *kb1 = P.num_kb; *slot = -1; }
+  t_decode(P, t, mb, nb);
 }
 __device__ __forceinline__ void named_sync(int id, int n) { asm volatile("bar.sync %0, %1;" ::"r"(id), "r"(n) : "memory"); }
 
@@ -203,8 +231,8 @@ __device__ __forceinline__ void tmem_ld32(uint32_t taddr, uint32_t* r) {
   asm volatile("tcgen05.wait::ld.sync.aligned;" ::: "memory");
 }
 
-template <int EPI, bool OUT_BF16>
-__global__ void __launch_bounds__(THREADS, 1)
+template <int EPI, bool OUT_BF16, bool AG = false>
+__global__ void __launch_bounds__(AG ? THREADS + AG_THREADS : THREADS, 1)
     gemm_kernel(const __grid_constant__ CUtensorMap mapA, const __grid_constant__ CUtensorMap mapB,
                 const __grid_constant__ Params P) {
   extern __shared__ __align__(1024) uint8_t smem_raw[];
@@ -215,6 +243,7 @@ __global__ void __launch_bounds__(THREADS, 1)
   uint64_t* bars = (uint64_t*)(smem + STAGES * STAGE_BYTES);
   // bars: full[STAGES], empty[STAGES], tmem_full[2], tmem_empty[2]; then the TMEM slot
   uint32_t* tmem_slot = (uint32_t*)(bars + 2 * STAGES + 4);
+  int64_t* s_koff = (int64_t*)(smem + STAGES * STAGE_BYTES + 256);    // AG: K-chunk offsets
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const uint32_t full0 = smem_u32(bars), empty0 = smem_u32(bars + STAGES);
   const uint32_t tfull0 = smem_u32(bars + 2 * STAGES), tempty0 = smem_u32(bars + 2 * STAGES + 2);
@@ -223,7 +252,7 @@ __global__ void __launch_bounds__(THREADS, 1)
     asm volatile("prefetch.tensormap [%0];" ::"l"((uint64_t)&mapA) : "memory");
     asm volatile("prefetch.tensormap [%0];" ::"l"((uint64_t)&mapB) : "memory");
     for (int s = 0; s < STAGES; ++s) {
-      mbar_init(full0 + 8 * s, 1);
+      mbar_init(full0 + 8 * s, AG ? 1 + AG_THREADS : 1);    // AG: TMA(B) + every gather thread
       mbar_init(empty0 + 8 * s, 1);
     }
     for (int a = 0; a < 2; ++a) {
@@ -247,17 +276,19 @@ __global__ void __launch_bounds__(THREADS, 1)
       // ===== TMA producer =====
       int stage = 0;
       uint32_t phase = 0;
-      for (int t = t_first(P); t < t_last(P); t += t_step(P)) {
-        int mb, nb;
-        t_decode(P, t, &mb, &nb);
+      for (int u = u_first(P); u < u_last(P); u += u_step(P)) {
+        int mb, nb, kb0, kb1, slot;
+        u_decode(P, u, &mb, &nb, &kb0, &kb1, &slot);
         const int m0 = mb * BM, n0 = nb * BN;
-        for (int kb = 0; kb < P.num_kb; ++kb) {
+        for (int kb = kb0; kb < kb1; ++kb) {
           mbar_wait(empty0 + 8 * stage, phase ^ 1);
           const uint32_t fb = full0 + 8 * stage;
-          mbar_expect_tx(fb, STAGE_BYTES);
+          mbar_expect_tx(fb, AG ? B_BYTES : STAGE_BYTES);
           const uint32_t a_dst = smem_u32(sA + stage * A_BYTES), b_dst = smem_u32(sB + stage * B_BYTES);
           const int k0 = kb * BK;
-          if (P.a_box) {               // implicit GEMM: one N-d box {64 k*, …1…, 128 g*}
+          if (AG) {
+            // A arrives from the gather warps
+          } else if (P.a_box) {               // implicit GEMM: one N-d box {64 k*, …1…, 128 g*}
             int cr[5];
             box_coords(P.abox, m0, k0, cr);
             tma_load_nd(a_dst, &mapA, fb, P.abox.rank, cr);
@@ -283,12 +314,14 @@ __global__ void __launch_bounds__(THREADS, 1)
       int stage = 0;
       uint32_t phase = 0;
       int it = 0;
-      for (int t = t_first(P); t < t_last(P); t += t_step(P), ++it) {
+      for (int u = u_first(P); u < u_last(P); u += u_step(P), ++it) {
+        int mb, nb, kb0, kb1, slot;
+        u_decode(P, u, &mb, &nb, &kb0, &kb1, &slot);
         const int acc = it & 1;
         mbar_wait(tempty0 + 8 * acc, ((it >> 1) & 1) ^ 1);
         tc_fence_after();
         const uint32_t d = tmem + acc * BN;
-        for (int kb = 0; kb < P.num_kb; ++kb) {
+        for (int kb = kb0; kb < kb1; ++kb) {
           mbar_wait(full0 + 8 * stage, phase);
           tc_fence_after();
           const uint32_t a0 = smem_u32(sA + stage * A_BYTES), b0 = smem_u32(sB + stage * B_BYTES);
@@ -298,7 +331,7 @@ __global__ void __launch_bounds__(THREADS, 1)
             // MN-major: +16 rows × 128 B = 2048 B per K step (LBO = next 64-wide MN atom)
             const uint64_t ad = P.a_mn_major ? sdesc(a0 + 2048 * k, 8192, 1024) : sdesc(a0 + 32 * k, 16, 1024);
             const uint64_t bd = P.b_mn_major ? sdesc(b0 + 2048 * k, 8192, 1024) : sdesc(b0 + 32 * k, 16, 1024);
-            mma_bf16(d, ad, bd, P.idesc, (kb | k) != 0);
+            mma_bf16(d, ad, bd, P.idesc, kb != kb0 || k != 0);
           }
           mma_commit(empty0 + 8 * stage);            // smem stage free once these MMAs retire
           if (++stage == STAGES) { stage = 0; phase ^= 1; }
@@ -306,6 +339,55 @@ __global__ void __launch_bounds__(THREADS, 1)
         mma_commit(tfull0 + 8 * acc);                 // accumulator ready for the epilogue
       }
     }
+  } else if (AG && warp >= THREADS / 32) {
+    // ===== A gather producer (warps 10..13): the A tile straight from the operand through
+    // its row / K-chunk offset tables with 16-byte cp.async into the SWIZZLE_128B K-major
+    // layout TMA would produce (16-B chunk c of row r at (c ^ (r & 7)) * 16), so no
+    // materialised im2col / permuted copy.  Thread → K chunk (gt & 7) of rows gt/8 + 16 i.
+    // A stage is published AG_LAG k-blocks later: wait_group, proxy fence, arrive.
+    const int gt = threadIdx.x - THREADS;
+    for (int i = gt; i < P.nkc; i += AG_THREADS) s_koff[i] = __ldg(P.aK + 8 * (int64_t)i);
+    named_sync(2, AG_THREADS);
+    const int ch = gt & 7, rb = gt >> 3;
+    int stage = 0;
+    uint32_t phase = 0;
+    int g = 0;                                   // k-blocks issued so far
+    for (int u = u_first(P); u < u_last(P); u += u_step(P)) {
+      int mb, nb, kb0, kb1, slot;
+      u_decode(P, u, &mb, &nb, &kb0, &kb1, &slot);
+      const int64_t m0 = (int64_t)mb * BM;
+      int64_t ro[8];
+#pragma unroll
+      for (int i = 0; i < 8; ++i) {
+        const int64_t m = m0 + rb + 16 * i;
+        ro[i] = m < P.M ? __ldg(P.aM + m) : -1;
+      }
+      for (int kb = kb0; kb < kb1; ++kb, ++g) {
+        mbar_wait(empty0 + 8 * stage, phase ^ 1);
+        const uint32_t base = smem_u32(sA + stage * A_BYTES);
+        const int kc = kb * (BK / 8) + ch;
+        const int64_t ko = kc < P.nkc ? s_koff[kc] : -1;
+#pragma unroll
+        for (int i = 0; i < 8; ++i) {
+          const int r = rb + 16 * i;
+          const uint32_t dst = base + r * 128 + ((ch ^ (r & 7)) << 4);
+          if (ro[i] >= 0 && ko >= 0) cp_async16(dst, P.Ag + ro[i] + ko);
+          else asm volatile("st.shared.v4.u32 [%0], {%1, %1, %1, %1};" ::"r"(dst), "r"(0) : "memory");
+        }
+        cp_async_commit();
+        if (g >= P.ag_lag) {
+          if (P.ag_lag == 1) cp_async_wait<1>();
+          else if (P.ag_lag == 2) cp_async_wait<2>();
+          else cp_async_wait<3>();
+          fence_proxy_async();
+          mbar_arrive(full0 + 8 * ((g - P.ag_lag) % STAGES));
+        }
+        if (++stage == STAGES) { stage = 0; phase ^= 1; }
+      }
+    }
+    cp_async_wait<0>();
+    fence_proxy_async();
+    for (int j = g - P.ag_lag < 0 ? 0 : g - P.ag_lag; j < g; ++j) mbar_arrive(full0 + 8 * (j % STAGES));
   } else {
     // ===== epilogue: warps 2..9; warp → TMEM lane quadrant (warp % 4) and a half of the
     // 256 accumulator columns (two warps per sub-partition hide the store latency) =====
@@ -314,10 +396,10 @@ __global__ void __launch_bounds__(THREADS, 1)
     const int row = quad * 32 + lane;
     int it = 0;
     int cached_nb = -1;
-    for (int t = t_first(P); t < t_last(P); t += t_step(P), ++it) {
+    for (int u = u_first(P); u < u_last(P); u += u_step(P), ++it) {
       const int acc = it & 1;
-      int mb, nbk;
-      t_decode(P, t, &mb, &nbk);
+      int mb, nbk, kb0, kb1, slot;
+      u_decode(P, u, &mb, &nbk, &kb0, &kb1, &slot);
       const int64_t m = (int64_t)mb * BM + row;
       const int64_t n0 = (int64_t)nbk * BN + half * (BN / 2);
       if (EPI == 1 && nbk != cached_nb) {
@@ -333,12 +415,48 @@ __global__ void __launch_bounds__(THREADS, 1)
       tc_fence_after();
       const bool mok = m < P.M;
       const int64_t crow = P.cbase + (EPI == 0 ? (mok ? m : 0) * P.ldc : __ldg(P.cM + (mok ? m : 0)));
+      // split-K tail (as in gemm2_kernel): splits 0..S-2 write a dense fp32 partial tile
+      // [128][256] and count their 8 warps in; the last split waits for them and folds
+      // p_0 + … + p_{S-2} + own in split order before the store
+      const bool split = slot >= 0;
+      const int ti = split ? slot / P.ssplit : 0;
+      const bool last = split && slot % P.ssplit == P.ssplit - 1;
+      unsigned* cnt = P.tail_cnt + 2 * ti;
+      const int64_t prel = (int64_t)row * BN + half * (BN / 2);
+      float* prow = (split && !last) ? P.part + (int64_t)slot * (BM * BN) + prel : nullptr;
+      if (last) {
+        if (lane == 0)
+          while (*((volatile unsigned*)cnt) < 8u * (unsigned)(P.ssplit - 1)) __nanosleep(64);
+        __syncwarp();
+        __threadfence();
+      }
 #pragma unroll 1
       for (int c = 0; c < BN / 64; ++c) {
         uint32_t r[32];
         tmem_ld32(tmem + ((uint32_t)(quad * 32) << 16) + acc * BN + half * (BN / 2) + c * 32, r);
         const int64_t nb = n0 + c * 32;
-        if (EPI == 0) {
+        if (last) {
+          const float* p0 = P.part + (int64_t)(ti * P.ssplit) * (BM * BN) + prel + c * 32;
+#pragma unroll
+          for (int j4 = 0; j4 < 8; ++j4) {
+            float4 a = *reinterpret_cast<const float4*>(p0 + 4 * j4);
+            for (int s2 = 1; s2 < P.ssplit - 1; ++s2) {
+              const float4 b = *reinterpret_cast<const float4*>(p0 + (int64_t)s2 * (BM * BN) + 4 * j4);
+              a.x += b.x; a.y += b.y; a.z += b.z; a.w += b.w;
+            }
+            r[4 * j4] = __float_as_uint(a.x + __uint_as_float(r[4 * j4]));
+            r[4 * j4 + 1] = __float_as_uint(a.y + __uint_as_float(r[4 * j4 + 1]));
+            r[4 * j4 + 2] = __float_as_uint(a.z + __uint_as_float(r[4 * j4 + 2]));
+            r[4 * j4 + 3] = __float_as_uint(a.w + __uint_as_float(r[4 * j4 + 3]));
+          }
+        }
+        if (prow) {
+          float4* dst = reinterpret_cast<float4*>(prow + c * 32);
+#pragma unroll
+          for (int j = 0; j < 8; ++j)
+            dst[j] = make_float4(__uint_as_float(r[4 * j]), __uint_as_float(r[4 * j + 1]), __uint_as_float(r[4 * j + 2]),
+                                 __uint_as_float(r[4 * j + 3]));
+        } else if (EPI == 0) {
           // row-major fp32 C: each thread writes 128 contiguous bytes of its row
           if (mok && nb + 32 <= P.N && ((crow + nb) & 3) == 0) {
             float4* dst = reinterpret_cast<float4*>(P.C + crow + nb);
@@ -370,6 +488,17 @@ __global__ void __launch_bounds__(THREADS, 1)
               }
             }
           }
+        }
+      }
+      if (split && !last) {            // publish this warp's part of the partial tile
+        __threadfence();
+        __syncwarp();
+        if (lane == 0) atomicAdd(cnt, 1u);
+      } else if (last) {               // 8 warps leave; the last one resets the counters
+        __syncwarp();
+        if (lane == 0 && atomicAdd(cnt + 1, 1u) == 7u) {
+          cnt[0] = 0u;
+          cnt[1] = 0u;
         }
       }
       tc_fence_before();
@@ -432,7 +561,6 @@ __device__ __forceinline__ void mma_commit_cg2(uint32_t bar) {
 __device__ __forceinline__ void mbar_arrive_cluster(uint32_t bar_cluster) {
   asm volatile("mbarrier.arrive.shared::cluster.b64 _, [%0];" ::"r"(bar_cluster) : "memory");
 }
-
 template <bool OUT_ROWMAJOR>
 __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(THREADS, 1)
     gemm2_kernel(const __grid_constant__ CUtensorMap mapA, const __grid_constant__ CUtensorMap mapB,
@@ -655,6 +783,7 @@ __global__ void __launch_bounds__(256) tail_combine_kernel(const __grid_constant
 }
 
 constexpr int MAX_TAIL_UNITS = 74;   // partial tiles reserved in the workspace (2-SM path)
+constexpr int MAX_TAIL_UNITS1 = 296; // 1-SM path: bound on tail units (partials sized per plan)
 
 // ---- operand normalisation pre-pass ---------------------------------------------------
 // An operand whose (MN, K) offsets are not 2-D linear (e.g. CCSD(T)'s t2 in output order,
@@ -837,6 +966,9 @@ struct T4State {
   t4::Layout2D a, b;
   t4::Params P;
   int cg = 1;      // 1: one SM per 128×256 tile; 2: SM pair per 256×256 tile
+  bool ag = false; // A staged by the kernel's gather warps (no A tensor map, no pre-pass)
+  int tail_parts = 0;   // 1-SM split-K tail: partial tiles in the workspace at tail_off
+  int grid1 = 0;        // its grid (the SM count at plan time: one tail unit per CTA)
   size_t tail_off = 0;
   // implicit-GEMM A map (a_box): TMA-order dims, byte strides, box
   int brank = 0;
@@ -918,9 +1050,27 @@ mdh_status prepare_t4(Plan* p) {
   const t4::Layout2D a_direct = t4::operand_layout(*p, c.md, c.nm, c.M, p->in[c.a_buf].acc[0], &w2, "A");
   // implicit GEMM is opt-in (tile knob implicit=1): measured slower than the gather
   // pre-pass on MCC conv5_1
-  const bool a_box = !(a_direct.ok && p->in[c.a_buf].acc[0].base % 8 == 0) && p->tiles.implicit == 1 && plan_box(p, s);
+  const bool a_2d = a_direct.ok && p->in[c.a_buf].acc[0].base % 8 == 0;
+  const bool a_box = !a_2d && p->tiles.implicit == 1 && plan_box(p, s);
   const t4::BoxGen box = s->P.abox;
-  if (a_box) {
+  // in-kernel gather (implicit 0 = auto or 2): A's K offsets in aligned runs of 8, so each
+  // 16-byte chunk of a swizzled A row is one cp.async
+  bool a_gather = false;
+  if (!a_2d && !a_box && (p->tiles.implicit == 0 || p->tiles.implicit == 2) && c.K % 8 == 0 &&
+      c.K / 8 <= t4::KOFF_MAX) {
+    std::vector<int64_t> tk = t4::table(*p, c.kd, c.nk, p->in[c.a_buf].acc[0]);
+    std::vector<int64_t> tm = t4::table(*p, c.md, c.nm, p->in[c.a_buf].acc[0]);
+    const int64_t base = p->in[c.a_buf].acc[0].base;
+    a_gather = true;
+    for (size_t i = 0; i < tk.size() && a_gather; i += 8) {
+      if ((tk[i] + base) % 8) a_gather = false;
+      for (int j = 1; j < 8 && a_gather; ++j)
+        if (tk[i + j] != tk[i] + j) a_gather = false;
+    }
+    for (size_t i = 0; i < tm.size() && a_gather; ++i)
+      if (tm[i] % 8) a_gather = false;
+  }
+  if (a_box || a_gather) {
     s->a = t4::Layout2D();
     s->a.ok = true;
   } else {
@@ -959,7 +1109,11 @@ mdh_status prepare_t4(Plan* p) {
   P.sched = P.c_rowmajor ? 0 : 1;
   // 2-SM pairs (cta_group::2, 256×256 tiles) for large row-major outputs (measured 1290 vs
   // 1170 TFLOP/s on MatMul 4096³); tile knob cluster=1 forces the 1-SM kernel
-  s->cg = (P.c_rowmajor && !P.out_bf16 && c.M >= 256 && c.N >= 256 && p->tiles.cluster != 1) ? 2 : 1;
+  // (the in-kernel A gather is a 1-SM kernel: a 2-SM version, whose peer CTA must publish
+  // its gathered half at cluster scope, measured 86-208 µs vs 83 µs on MCC conv5_1)
+  s->ag = a_gather;
+  P.nkc = (int)(c.K / 8);
+  s->cg = (!a_gather && P.c_rowmajor && !P.out_bf16 && c.M >= 256 && c.N >= 256 && p->tiles.cluster != 1) ? 2 : 1;
   if (s->cg == 2) {
     P.tiles_m = (int)((c.M + 255) / 256);
     P.tiles_n = (int)((c.N + 255) / 256);
@@ -969,9 +1123,37 @@ mdh_status prepare_t4(Plan* p) {
     ws = (ws + 255) / 256 * 256;
     s->tail_off = ws;
     ws += (size_t)t4::MAX_TAIL_UNITS * 65536 * sizeof(float) + 2 * t4::MAX_TAIL_UNITS * sizeof(unsigned) + 256;
+  } else {
+    // 1-SM split-K tail: the T mod C tiles of the last, partial wave split along K over
+    // the idle SMs (S units each) — tile knob split=S, or automatically when the partial
+    // wave is a large share of a K-deep contraction (MCC conv5_1: 196 tiles on 148 SMs)
+    int dev = p->device, sms = 148;
+    if (cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev) != cudaSuccess || sms <= 0) {
+      cudaGetLastError();
+      sms = 148;
+    }
+    const int T = P.num_tiles, C = std::max(1, std::min(T, sms)), R = T / C, Tr = T - R * C;
+    int S = 1;
+    if (Tr > 0) {
+      const int cap = std::min({C / Tr, P.num_kb / 4, t4::MAX_TAIL_UNITS1 / Tr});
+      if (p->tiles.split > 1) S = std::min(p->tiles.split, cap);
+      // (no automatic split: on MCC conv5_1 split 2/3/4 measured 84/92/92 µs vs 84 whole)
+    }
+    if (S >= 2) {
+      P.sched = 0;
+      P.nfull = T - Tr;
+      P.ssplit = S;
+      P.nunits = P.nfull + Tr * S;
+      ws = (ws + 255) / 256 * 256;
+      s->tail_off = ws;
+      ws += (size_t)Tr * S * t4::BM * t4::BN * sizeof(float) + 2 * (size_t)Tr * sizeof(unsigned) + 256;
+      s->tail_parts = Tr * S;
+      s->grid1 = C;
+    }
   }
   p->tmaps = s;
-  p->t4_variant = 1 + (s->a.permuted ? 2 : 0) + (s->b.permuted ? 4 : 0) + (s->cg == 2 ? 8 : 0) + (a_box ? 16 : 0);
+  p->t4_variant = 1 + (s->a.permuted ? 2 : 0) + (s->b.permuted ? 4 : 0) + (s->cg == 2 ? 8 : 0) + (a_box ? 16 : 0) +
+                  (a_gather ? 32 : 0);
   p->ws_kernel = ws;
   p->tiles.bm = s->cg == 2 ? 256 : t4::BM;
   p->tiles.bn = t4::BN;
@@ -1081,10 +1263,16 @@ mdh_status launch_t4(const Plan& p, const void* const* in, void* const* out, voi
                     strides, box, estr, CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_128B,
                     CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
     if (r != CUDA_SUCCESS) { set_error("cuTensorMapEncodeTiled (implicit GEMM) failed (%d)", (int)r); return MDH_ERR_CUDA; }
+  } else if (s->ag) {
+    if ((uintptr_t)A % 16) { set_error("T4 gather: A buffer not 16-byte aligned"); return MDH_ERR_INVALID_ARG; }
+    P.Ag = A;
+    P.aM = (const int64_t*)(dc + p.tab_off[0]);
+    P.aK = (const int64_t*)(dc + p.tab_off[1]);
   } else if (s->a.mn_major) MDH_TRY(make_map(&ma, A, c.M, c.K, s->a.ld, 64, 64));
   else MDH_TRY(make_map(&ma, A, c.K, c.M, s->a.ld, 64, 128));
   if (s->b.mn_major) MDH_TRY(make_map(&mb, B, c.N, c.K, s->b.ld, 64, 64));
   else MDH_TRY(make_map(&mb, B, c.K, c.N, s->b.ld, 64, s->cg == 2 ? 128 : 256));
+  if (s->ag) ma = mb;
   static std::once_flag attr_once;
   static cudaError_t attr_err = cudaSuccess;
   std::call_once(attr_once, [] {
@@ -1094,11 +1282,18 @@ mdh_status launch_t4(const Plan& p, const void* const* in, void* const* out, voi
       cudaError_t e = cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, t4::SMEM_BYTES);
       if (e != cudaSuccess) attr_err = e;
     }
+    const void* kg[3] = {(const void*)t4::gemm_kernel<0, false, true>, (const void*)t4::gemm_kernel<1, false, true>,
+                         (const void*)t4::gemm_kernel<1, true, true>};
+    for (const void* k : kg) {
+      cudaError_t e = cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, t4::SMEM_AG_BYTES);
+      if (e != cudaSuccess) attr_err = e;
+    }
     const void* k2[2] = {(const void*)t4::gemm2_kernel<true>, (const void*)t4::gemm2_kernel<false>};
     for (const void* k : k2) {
       cudaError_t e = cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, t4::SMEM2_BYTES);
       if (e != cudaSuccess) attr_err = e;
     }
+
   });
   MDH_CUDA(attr_err);
   int dev = 0, sms = 148;
@@ -1128,7 +1323,20 @@ mdh_status launch_t4(const Plan& p, const void* const* in, void* const* out, voi
     t4::gemm2_kernel<true><<<grid2, t4::THREADS, t4::SMEM2_BYTES, st>>>(ma, mb, P);
     return post_launch("t4_gemm2_kernel");
   }
-  const int grid = std::min(P.num_tiles, sms);
+  int grid = std::min(P.num_tiles, sms);
+  if (s->tail_parts) {
+    grid = s->grid1;
+    P.part = (float*)((char*)ws + s->tail_off);
+    P.tail_cnt = (unsigned*)((char*)ws + s->tail_off + (size_t)s->tail_parts * t4::BM * t4::BN * sizeof(float));
+  }
+  if (s->ag) {
+    P.ag_lag = 2;   // measured on MCC conv5_1: lag 1 / 2 / 3 → 89 / 83 / 130 µs
+    constexpr int TG = t4::THREADS + t4::AG_THREADS;
+    if (P.c_rowmajor && !P.out_bf16) t4::gemm_kernel<0, false, true><<<grid, TG, t4::SMEM_AG_BYTES, st>>>(ma, mb, P);
+    else if (!P.out_bf16) t4::gemm_kernel<1, false, true><<<grid, TG, t4::SMEM_AG_BYTES, st>>>(ma, mb, P);
+    else t4::gemm_kernel<1, true, true><<<grid, TG, t4::SMEM_AG_BYTES, st>>>(ma, mb, P);
+    return post_launch("t4_gemm_kernel_ag");
+  }
   if (P.c_rowmajor && !P.out_bf16) t4::gemm_kernel<0, false><<<grid, t4::THREADS, t4::SMEM_BYTES, st>>>(ma, mb, P);
   else if (!P.out_bf16) t4::gemm_kernel<1, false><<<grid, t4::THREADS, t4::SMEM_BYTES, st>>>(ma, mb, P);
   else t4::gemm_kernel<1, true><<<grid, t4::THREADS, t4::SMEM_BYTES, st>>>(ma, mb, P);

@@ -393,21 +393,39 @@ def test_mcc_bf16_tcgen05(cfg):
     assert_close_full(spec, x, got, 1e-2, kind="scale")
 
 
-@pytest.mark.parametrize("tile", ["implicit=1", "cluster=2"])
+@pytest.mark.parametrize("tile", ["implicit=1", "implicit=2", "implicit=3", "cluster=2"])
 def test_t4_variants_parity(tile):
-    """The opt-in T4 variants: implicit-GEMM N-d TMA operand (MCC) and 2-SM pairs (MatMul)."""
-    if tile == "implicit=1":
+    """T4 A-operand variants on MCC (1: implicit-GEMM N-d TMA box, 2: in-kernel cp.async
+    gather, 3: gather pre-pass) and 2-SM pairs on MatMul."""
+    if tile.startswith("implicit"):
         spec = S.mcc(128, 7, 7, 128, 3, 3, 128, "bf16")
         x = G.mcc_inputs(spec)
         got, p = run_gpu(spec, x, force_tile=tile)
-        assert p.describe()["t4_variant"] & 16
-        assert_close_full(spec, x, got, 1e-2, kind="scale") if False else assert_close_points(spec, x, got, 1e-2, n=4000, kind="scale")
+        v = p.describe()["t4_variant"]
+        assert v & {"implicit=1": 16, "implicit=2": 32, "implicit=3": 2}[tile], v
+        assert_close_points(spec, x, got, 1e-2, n=4000, kind="scale")
     else:
         spec = S.matmul(1024, 768, 640, "bf16")
         x = G.matmul_inputs(1024, 768, 640, "bf16", "positive")
         got, p = run_gpu(spec, x, force_tile=tile)
         assert p.describe()["t4_variant"] & 8
         assert_close_full(spec, x, got, 1e-2, kind="rel")
+
+
+@pytest.mark.parametrize("shape,tile,out", [((2560, 2048, 1024), "cluster=1,split=3", "f32"),
+                                            ((2500, 2000, 1000), "cluster=1,split=2", "f32"),
+                                            ((2500, 2000, 1000), "split=4", "bf16")])
+def test_t4_split_tail_1sm(shape, tile, out):
+    """1-SM split-K tail: the partial last wave's tiles split along K (fused fixup in split
+    order), row-major (EPI 0) and table-scatter bf16 (EPI 1) epilogues, ragged M/N/K."""
+    M, N, K = shape
+    spec = S.matmul(M, N, K, "bf16", out_dtype=out)
+    x = G.matmul_inputs(M, N, K, "bf16", "positive")
+    plan = None
+    for _ in range(2):                      # second run: the tail counters were reset
+        got, plan = run_gpu(spec, x, plan=plan, force_tile=tile)
+        assert not plan.describe()["t4_variant"] & 8
+        assert_close_points(spec, x, got, 1e-2, n=20000, kind="rel")
 
 
 def test_mcc_bf16_config_sampled():

@@ -28,6 +28,8 @@ def cases():
         "t4_2sm": (lambda: S.matmul(512, 512, 256, "bf16"), "positive", None),
         "t4_gather": (lambda: S.ccsd_sd1(2, 3, "bf16"), "signed", None),
         "t4_split": (lambda: S.matmul(1280, 768, 512, "bf16"), "positive", "split=3"),
+        "t4_ag": (lambda: S.mcc(4, 7, 7, 64, 3, 3, 16, "bf16"), "positive", None),
+        "t4_split1": (lambda: S.matmul(2500, 2000, 512, "bf16", out_dtype="bf16"), "positive", "split=2"),
         "t5": (lambda: S.prl(300, 2000), "prl", None),
         "t6": (lambda: S.prefix_sum([3, 9000], 1), "positive", None),
         "combine": (lambda: S.dot(5000, "i32"), "virtual", None),
