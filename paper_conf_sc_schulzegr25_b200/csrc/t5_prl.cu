@@ -8,15 +8,18 @@
 // order-preserving mapping required by the non-commutative paper rule, reading C-2).
 // f (reading C-18): an 8-bit agreement mask from 8 u32 equality tests; the fold only
 // needs the ORDER of (id==14, weight) which the plan precomputes per mask as a dense
-// rank (ties equal), so a pair costs the 8 compares, one conflict-free byte lookup
-// (the rank table is replicated per lane/bank) and a lexicographic compare with the
-// running best (rank, match_id).  The fp64 weight Σ_k (bit_k ? wa_k : wd_k), summed in
+// rank (ties equal), so a pair costs the 8 compares — each selecting its bit already
+// scaled to the table stride and summed onto the lane's table base, so the sum IS the
+// shared-memory address — one conflict-free lookup (the rank table is replicated per
+// lane/bank) and one compare with the running best rank; match_id is read and compared
+// only when the ranks tie (rare once the best has risen).  The fp64 weight Σ_k (bit_k ? wa_k : wd_k), summed in
 // field order, and id_measure are produced only for the final best record.
 // The reduction dim is split over CTAs when N alone cannot fill the GPU (orientation
 // B, 2^14 × 2^20; reading C-20): partial records [S][N] are folded in split order by
 // a combine kernel (A7), lhs = lower range.
 #include <algorithm>
 #include <vector>
+#include <mutex>
 
 #include "kcommon.cuh"
 #include "prl_common.cuh"
@@ -24,7 +27,8 @@
 namespace mdh {
 
 constexpr int T5_THREADS = 256;
-constexpr int T5_R = 4;           // new records per thread
+constexpr int T5_R = 4;           // new records per thread (T5_R8 = 8 when N fills the GPU)
+constexpr int T5_R8 = 8;
 constexpr int T5_TILE = 512;      // DB records per smem tile
 
 struct T5Params {
@@ -35,7 +39,7 @@ struct T5Params {
   int64_t dbase[9], dL[9];        // db field k (k=8: id) of record i at dbase + dL*i
   int64_t N, I, ichunk;
   int S, op;
-  const uint8_t* rank32;          // [64][32] words: byte (mask&3) of word (mask>>2)*32+lane
+  const uint32_t* rank32;         // [256][32] words: rank of mask m at m*32 + lane
   const double* wtab;             // [256] fp64 weights
   // outputs: final (through ω) or partials [S][N]
   long long* oid;
@@ -47,12 +51,36 @@ struct T5Params {
   int32_t* pm;
 };
 
+// shared-memory address of the rank of the agreement mask of new record v and DB record
+// (lo, hi): base + Σ_k [v_k == db_k] · (128 << k) — compare + select per field, the
+// selects summed three at a time
+__device__ __forceinline__ uint32_t mask_addr(const uint32_t* v, const uint4& lo, const uint4& hi, uint32_t base) {
+  // compare, then a predicated add of the scaled bit onto the running address: 2 ops/field
+  uint32_t a = base;
+  asm("{\n\t.reg .pred q0, q1, q2, q3, q4, q5, q6, q7;\n\t"
+      "setp.eq.u32 q0, %1, %9;\n\tsetp.eq.u32 q1, %2, %10;\n\t"
+      "setp.eq.u32 q2, %3, %11;\n\tsetp.eq.u32 q3, %4, %12;\n\t"
+      "setp.eq.u32 q4, %5, %13;\n\tsetp.eq.u32 q5, %6, %14;\n\t"
+      "setp.eq.u32 q6, %7, %15;\n\tsetp.eq.u32 q7, %8, %16;\n\t"
+      "@q0 add.u32 %0, %0, 128;\n\t@q1 add.u32 %0, %0, 256;\n\t"
+      "@q2 add.u32 %0, %0, 512;\n\t@q3 add.u32 %0, %0, 1024;\n\t"
+      "@q4 add.u32 %0, %0, 2048;\n\t@q5 add.u32 %0, %0, 4096;\n\t"
+      "@q6 add.u32 %0, %0, 8192;\n\t@q7 add.u32 %0, %0, 16384;\n\t}"
+      : "+r"(a)
+      : "r"(v[0]), "r"(v[1]), "r"(v[2]), "r"(v[3]), "r"(v[4]), "r"(v[5]), "r"(v[6]), "r"(v[7]), "r"(lo.x), "r"(lo.y),
+        "r"(lo.z), "r"(lo.w), "r"(hi.x), "r"(hi.y), "r"(hi.z), "r"(hi.w));
+  return a;
+}
+
+template <int R>
 __global__ void __launch_bounds__(T5_THREADS) t5_kernel(const __grid_constant__ T5Params P) {
+  constexpr int T5_R = R;
   __shared__ __align__(16) uint32_t sf[T5_TILE][8];
   __shared__ long long sid[T5_TILE];
-  __shared__ uint32_t srank[64 * 32];
+  extern __shared__ uint32_t srank[];     // [256][32], dynamic (32 KB)
   const int tid = threadIdx.x, lane = tid & 31;
-  for (int k = tid; k < 64 * 32; k += T5_THREADS) srank[k] = ((const uint32_t*)P.rank32)[k];
+  for (int k = tid; k < 256 * 32; k += T5_THREADS) srank[k] = P.rank32[k];
+  const uint32_t lanebase = (uint32_t)__cvta_generic_to_shared(srank) + 4u * lane;
   const int64_t nblk = (P.N + T5_THREADS * T5_R - 1) / (T5_THREADS * T5_R);
   const int64_t bn = blockIdx.x % nblk;
   const int s = (int)(blockIdx.x / nblk);
@@ -89,22 +117,39 @@ __global__ void __launch_bounds__(T5_THREADS) t5_kernel(const __grid_constant__ 
       const uint4 lo = *reinterpret_cast<const uint4*>(&sf[j][0]);
       const uint4 hi = *reinterpret_cast<const uint4*>(&sf[j][4]);
       const long long id = sid[j];
+      if (paper) {
+        const long long id = sid[j];
 #pragma unroll
-      for (int r = 0; r < T5_R; ++r) {
-        uint32_t m = (uint32_t)(nv[r][0] == lo.x) | ((uint32_t)(nv[r][1] == lo.y) << 1) |
-                     ((uint32_t)(nv[r][2] == lo.z) << 2) | ((uint32_t)(nv[r][3] == lo.w) << 3) |
-                     ((uint32_t)(nv[r][4] == hi.x) << 4) | ((uint32_t)(nv[r][5] == hi.y) << 5) |
-                     ((uint32_t)(nv[r][6] == hi.z) << 6) | ((uint32_t)(nv[r][7] == hi.w) << 7);
-        if (paper) {
+        for (int r = 0; r < T5_R; ++r) {
+          uint32_t m = (uint32_t)(nv[r][0] == lo.x) | ((uint32_t)(nv[r][1] == lo.y) << 1) |
+                       ((uint32_t)(nv[r][2] == lo.z) << 2) | ((uint32_t)(nv[r][3] == lo.w) << 3) |
+                       ((uint32_t)(nv[r][4] == hi.x) << 4) | ((uint32_t)(nv[r][5] == hi.y) << 5) |
+                       ((uint32_t)(nv[r][6] == hi.z) << 6) | ((uint32_t)(nv[r][7] == hi.w) << 7);
           // Listing 11: res = lhs if (lhs.id==14 && rhs.id!=14) else rhs
           const bool m14 = m == 0xFFu;
           const bool keep = b14[r] && !m14;
           if (!keep) { bid[r] = id; bmask[r] = m; b14[r] = m14; brank[r] = 0; }
-        } else {
-          const uint32_t word = srank[(m >> 2) * 32 + lane];
-          const int rk = (int)((word >> ((m & 3u) * 8u)) & 0xFFu);
-          const bool take = rk > brank[r] || (rk == brank[r] && id > bid[r]);
-          if (take) { brank[r] = rk; bid[r] = id; bmask[r] = m; }
+        }
+      } else {
+        uint32_t a[T5_R];
+        int rk[T5_R];
+        bool any = false;
+#pragma unroll
+        for (int r = 0; r < T5_R; ++r) {
+          a[r] = mask_addr(nv[r], lo, hi, lanebase);
+          asm("ld.shared.u32 %0, [%1];" : "=r"(rk[r]) : "r"(a[r]));
+        }
+#pragma unroll
+        for (int r = 0; r < T5_R; ++r) any |= rk[r] >= brank[r];
+        if (any) {                       // some rank reached the running best: tie-break on id
+          const long long id = sid[j];
+#pragma unroll
+          for (int r = 0; r < T5_R; ++r)
+            if (rk[r] > brank[r] || (rk[r] == brank[r] && id > bid[r])) {
+              brank[r] = rk[r];
+              bid[r] = id;
+              bmask[r] = (a[r] - lanebase) >> 7;
+            }
         }
       }
     }
@@ -184,23 +229,42 @@ mdh_status prepare_t5(Plan* p) {
     if (q > 0 && key_less(order[q - 1], order[q])) ++r;
     rank[order[q]] = (uint8_t)r;
   }
-  uint32_t rep[64 * 32];
-  for (int w = 0; w < 64; ++w) {
-    uint32_t word = (uint32_t)rank[4 * w] | ((uint32_t)rank[4 * w + 1] << 8) | ((uint32_t)rank[4 * w + 2] << 16) |
-                    ((uint32_t)rank[4 * w + 3] << 24);
-    for (int l = 0; l < 32; ++l) rep[w * 32 + l] = word;
-  }
+  std::vector<uint32_t> rep(256 * 32);
+  for (int m = 0; m < 256; ++m)
+    for (int l = 0; l < 32; ++l) rep[m * 32 + l] = rank[m];
   p->host_const.clear();
-  p->tab_off[0] = add_const(p, rep, sizeof(rep));
+  p->tab_off[0] = add_const(p, rep.data(), rep.size() * sizeof(uint32_t));
   p->tab_off[1] = add_const(p, W, sizeof(W));
-  // split the DB dim when N alone cannot fill the GPU
   int64_t N = nd >= 0 ? p->size[nd] : 1, I = id >= 0 ? p->size[id] : 1;
-  int64_t nblk = (N + T5_THREADS * T5_R - 1) / (T5_THREADS * T5_R);
+  // 4 new records per thread (8: tile knob vec=8 — measured 1147 vs 1466 Gpairs/s on 2^20×2^14)
+  int Rn = T5_R;
+  if (p->tiles.source.find("forced") != std::string::npos && p->tiles.vec == 8) Rn = T5_R8;
+  p->tiles.vec = Rn;
+  int64_t nblk = (N + T5_THREADS * Rn - 1) / (T5_THREADS * Rn);
+  // split the DB dim when N alone gives less than two waves of CTAs, choosing S so the
+  // CTAs fill whole waves: time ∝ ceil(nblk·S / slots) / S (slots = SMs × resident CTAs),
+  // smallest S on ties, I-chunks of at least one tile.  (With ≥ 2 waves the partial last
+  // wave costs little — resident CTAs share an SM's issue slots — and splitting measured
+  // slower: 2^20×2^14 at S = 13 took 12.96 ms vs 11.72 ms unsplit.)
+  int sms = 148, per_sm = 2;
+  if (cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, p->device) != cudaSuccess) { cudaGetLastError(); sms = 148; }
+  if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, Rn == T5_R8 ? (const void*)t5_kernel<T5_R8> : (const void*)t5_kernel<T5_R>,
+                                                    T5_THREADS, 256 * 32 * 4) != cudaSuccess || per_sm < 1) {
+    cudaGetLastError();
+    per_sm = 2;
+  }
+  const int64_t slots = (int64_t)sms * per_sm;
+  const int smax = (int)std::max<int64_t>(1, std::min<int64_t>(64, (I + T5_TILE - 1) / T5_TILE));
   int S = 1;
-  if (p->tiles.split > 0) S = p->tiles.split;
-  else if (nblk < 148 * 4) S = (int)std::min<int64_t>((148 * 4 + nblk - 1) / nblk, 64);
-  S = (int)std::max<int64_t>(1, std::min<int64_t>(S, (I + T5_TILE - 1) / T5_TILE));
-  if (S > 64) S = 64;
+  if (p->tiles.split > 0) {
+    S = std::min(p->tiles.split, smax);
+  } else if (nblk < 2 * slots) {
+    double best = 1e30;
+    for (int c = 1; c <= smax; ++c) {
+      const double t = (double)((nblk * c + slots - 1) / slots) / c;
+      if (t < best * (1 - 1e-9)) { best = t; S = c; }
+    }
+  }
   p->tiles.split = S;
   p->ws_kernel = S > 1 ? (size_t)S * N * (8 + 8 + 4) + 1024 : 0;
   return MDH_OK;
@@ -228,7 +292,7 @@ mdh_status launch_t5(const Plan& p, const void* const* in, void* const* out, voi
   P.S = p.tiles.split;
   P.ichunk = (P.I + P.S - 1) / P.S;
   P.op = p.redop == MDH_CC ? MDH_PW_PRL_ARGMAX : p.redop;
-  P.rank32 = (const uint8_t*)(dc + p.tab_off[0]);
+  P.rank32 = (const uint32_t*)(dc + p.tab_off[0]);
   P.wtab = (const double*)(dc + p.tab_off[1]);
   P.oid = (long long*)out[0];
   P.ow = (double*)out[1];
@@ -241,8 +305,19 @@ mdh_status launch_t5(const Plan& p, const void* const* in, void* const* out, voi
   P.pid = (long long*)w;
   P.pw = (double*)(w + (size_t)P.S * P.N * 8);
   P.pm = (int32_t*)(w + (size_t)P.S * P.N * 16);
-  const int64_t nblk = (P.N + T5_THREADS * T5_R - 1) / (T5_THREADS * T5_R);
-  t5_kernel<<<(unsigned)(nblk * P.S), T5_THREADS, 0, st>>>(P);
+  const int Rn = p.tiles.vec == T5_R8 ? T5_R8 : T5_R;
+  const int64_t nblk = (P.N + T5_THREADS * Rn - 1) / (T5_THREADS * Rn);
+  constexpr int SMEM_RANK = 256 * 32 * 4;
+  static std::once_flag once;
+  static cudaError_t aerr = cudaSuccess;
+  std::call_once(once, [] {
+    cudaError_t e1 = cudaFuncSetAttribute((const void*)t5_kernel<T5_R>, cudaFuncAttributeMaxDynamicSharedMemorySize, SMEM_RANK);
+    cudaError_t e2 = cudaFuncSetAttribute((const void*)t5_kernel<T5_R8>, cudaFuncAttributeMaxDynamicSharedMemorySize, SMEM_RANK);
+    aerr = e1 != cudaSuccess ? e1 : e2;
+  });
+  MDH_CUDA(aerr);
+  if (Rn == T5_R8) t5_kernel<T5_R8><<<(unsigned)(nblk * P.S), T5_THREADS, SMEM_RANK, st>>>(P);
+  else t5_kernel<T5_R><<<(unsigned)(nblk * P.S), T5_THREADS, SMEM_RANK, st>>>(P);
   MDH_TRY(post_launch("t5_kernel"));
   if (P.S > 1) {
     t5_combine<<<(unsigned)std::min<int64_t>((P.N + 255) / 256, 148 * 16), 256, 0, st>>>(P);

@@ -221,6 +221,20 @@ def test_prl_full(NI, op):
     assert_close_full(spec, ins, got, 0, kind="exact")
 
 
+@pytest.mark.parametrize("R", [4, 8])
+def test_prl_ties_full(R):
+    """Rank ties (weights with equal sums for different masks, duplicated DB ids) through
+    the id tie-break path, both register blockings (tile knob vec)."""
+    N, I = 3000, 2500
+    ins = G.prl_inputs(N, I, seed_base=5900)
+    ins[16] = (ins[16] % 97).astype(np.int64)          # many equal ids
+    wa, wd = [1.0, 1.0, 2.0, 2.0, 0.5, 0.5, 1.5, 1.5], [-1.0] * 8
+    for op in ("PW_PRL_ARGMAX", "PW_PRL_PAPER"):
+        spec = S.prl(N, I, op, weights=(wa, wd))
+        got, p = run_gpu(spec, ins, force_tile=f"vec={R}")
+        assert_close_full(spec, ins, got, 0, kind="exact")
+
+
 @pytest.mark.parametrize("NI", [(1 << 20, 1 << 14), (1 << 14, 1 << 20)])
 def test_prl_config_sampled(NI):
     N, I = NI
