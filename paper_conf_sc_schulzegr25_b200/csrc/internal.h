@@ -65,6 +65,7 @@ struct Tiles {
   int stages = 4;
   int vec = 4;
   int zchunk = 32;
+  int seg = 0;                        // T6: elements per L2-resident scan segment (0 = auto)
   int per_thread = 1;
   int cluster = 1;
   int implicit = 0;                   // T4 A operand when not 2-D: 0 auto, 1 N-d TMA box (implicit

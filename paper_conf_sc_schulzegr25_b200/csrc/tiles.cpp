@@ -140,6 +140,7 @@ void apply(Tiles* t, const std::string& k, double v) {
   else if (k == "stages") t->stages = iv;
   else if (k == "vec") t->vec = iv;
   else if (k == "zchunk") t->zchunk = iv;
+  else if (k == "seg") t->seg = iv;
   else if (k == "per_thread") t->per_thread = iv;
   else if (k == "cluster") t->cluster = iv;
   else if (k == "implicit") t->implicit = iv;

@@ -71,6 +71,33 @@ def test_gpu_prefix_sum(shape, dim, dt):
 
 
 @gpu
+@pytest.mark.parametrize("shape,dt,tile", [([3, 200000], "i32", None), ([3, 100003], "f32", None),
+                                           ([2, 300001], "f64", "seg=4096"), ([1 << 22], "i64", "seg=65536"),
+                                           ([1 << 22], "u32", None), ([5, 65536 * 3 + 4096 * 5 + 1], "f32", None),
+                                           ([(1 << 24) + 12345], "f32", None), ([3, 100003], "f32", "seg=8192")])
+def test_gpu_single_pass_scan(shape, dt, tile):
+    """Long rows take a single-pass scan: the tree scan (default; per-row tree of tile
+    aggregates) or the segmented one (tile knob seg): aligned and misaligned row starts,
+    ragged tile counts, several rows, integer wrap-around exact, repeatable."""
+    from gpu_util import run_gpu
+    spec = S.prefix_sum(shape, len(shape) - 1, dt)
+    x = G.gen_inputs(spec, 6150, "signed" if dt in ("f32", "f64") else "positive")
+    got, p = run_gpu(spec, x, force_tile=tile)
+    assert p.template == "T6_prefix_scan" and (p.describe()["tiles"]["seg"] > 0) == (tile is not None)
+    x0 = x[0].reshape(shape)
+    if dt in ("f32", "f64"):
+        ref = np.cumsum(x0.astype(np.float64), axis=-1)
+        scale = np.cumsum(np.abs(x0.astype(np.float64)), axis=-1)
+        assert np.max(np.abs(got[0].reshape(shape) - ref) / scale) <= (1e-4 if dt == "f32" else 1e-12)
+    else:   # two's-complement wrap: cumsum in the same width is exact
+        ref = np.cumsum(x0, axis=-1, dtype=x0.dtype)
+        assert np.array_equal(got[0].reshape(shape), ref)
+    for _ in range(2):                         # repeatable (deterministic association, epochs)
+        got2, _ = run_gpu(spec, x, plan=p)
+        assert np.array_equal(got[0], got2[0])
+
+
+@gpu
 @pytest.mark.parametrize("IJ", [(64, 37), (1000, 5000), (4096, 8192)])
 def test_gpu_mbbs(IJ):
     from gpu_util import assert_close_full, run_gpu
