@@ -24,7 +24,13 @@ def main():
     pk = bench.peaks()
     flush = bench.L2Flush(dev)
     for name in a.workloads:
-        w = bench.workload(name)
+        if name.startswith("mm:"):          # ad-hoc bf16 GEMM shape "mm:M,N,K"
+            from mdh_workloads import specs as S, gen as G
+            M, N, K = (int(v) for v in name[3:].split(","))
+            w = dict(spec=S.matmul(M, N, K, "bf16"), inputs=lambda M=M, N=N, K=K: G.matmul_inputs(M, N, K, "bf16"),
+                     work=2.0 * M * N * K, unit="TFLOP/s", scale=1e12, bound="tensor", dtype="bf16")
+        else:
+            w = bench.workload(name)
         plan = Plan(w["spec"], force_tile=a.force_tile)
         tin = [to_device(x, b["dtype"], dev) for x, b in zip(w["inputs"](), w["spec"]["inputs"])]
         outs = plan.empty_outputs(dev)
