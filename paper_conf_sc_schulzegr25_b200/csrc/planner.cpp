@@ -256,6 +256,25 @@ static bool group_contraction(Plan* p) {
   by_out_stride(c.md, c.nm);
   by_out_stride(c.nd, c.nn);
   by_out_stride(c.zd, c.nz);
+  // orientation: the output's most contiguous dim goes to the N group (TMEM columns in T4,
+  // the thread-x direction in T3), so a thread's consecutive accumulators are consecutive
+  // output elements and the epilogue stores vectors.  f = MUL is commutative (x0·x1 =
+  // x1·x0 exactly), so A/B may swap (CCSD(T): t3's unit-stride p4 is a t2 dim)
+  auto min_stride = [&](const int* dims, int n) {
+    int64_t s = INT64_MAX;
+    for (int t = 0; t < n; ++t) s = std::min(s, Co.L[dims[t]] < 0 ? -Co.L[dims[t]] : Co.L[dims[t]]);
+    return s;
+  };
+  if (min_stride(c.md, c.nm) < min_stride(c.nd, c.nn)) {
+    int tmp[MDH_MAX_D];
+    std::copy(c.md, c.md + c.nm, tmp);
+    std::copy(c.nd, c.nd + c.nn, c.md);
+    std::copy(tmp, tmp + c.nm, c.nd);
+    std::swap(c.nm, c.nn);
+    std::swap(c.M, c.N);
+    c.a_buf = 1;
+    c.b_buf = 0;
+  }
   p->con = c;
   return true;
 }
@@ -501,9 +520,9 @@ std::string describe_plan(const Plan& p) {
     add(", \"contraction\": {\"Z\": %lld, \"M\": %lld, \"N\": %lld, \"K\": %lld, \"nm\": %d, \"nn\": %d, \"nk\": %d, \"nz\": %d}",
         (long long)p.con.Z, (long long)p.con.M, (long long)p.con.N, (long long)p.con.K, p.con.nm, p.con.nn, p.con.nk, p.con.nz);
   add(", \"tiles\": {\"threads\": %d, \"bm\": %d, \"bn\": %d, \"bk\": %d, \"split\": %d, \"stages\": %d, \"vec\": %d, "
-      "\"zchunk\": %d, \"per_thread\": %d, \"cluster\": %d, \"implicit\": %d, \"seg\": %d, \"source\": \"%s\"}",
+      "\"zchunk\": %d, \"per_thread\": %d, \"cluster\": %d, \"implicit\": %d, \"seg\": %d, \"epi\": %d, \"source\": \"%s\"}",
       p.tiles.threads, p.tiles.bm, p.tiles.bn, p.tiles.bk, p.tiles.split, p.tiles.stages, p.tiles.vec,
-      p.tiles.zchunk, p.tiles.per_thread, p.tiles.cluster, p.tiles.implicit, p.tiles.seg, p.tiles.source.c_str());
+      p.tiles.zchunk, p.tiles.per_thread, p.tiles.cluster, p.tiles.implicit, p.tiles.seg, p.tiles.epi, p.tiles.source.c_str());
   add(", \"t4_variant\": %d", p.t4_variant);
   add(", \"workspace\": %zu, \"world\": %d, \"rank\": %d, \"shard_dim\": %d, \"shard_is_red\": %s, "
       "\"shard_start\": %lld, \"shard_len\": %lld}",

@@ -78,10 +78,14 @@ struct Params {
   const int64_t* aK;                // offA_K table (every 8th entry is a chunk start)
   int nkc;                          // K / 8 chunk offsets staged in shared memory
   int ag_lag;                       // k-blocks between issuing a stage and publishing it (1..3)
+  // bulk-run epilogue (EPI 3): N-tile = 2 output runs of bn/2 contiguous elements
+  int bn;                           // N-tile width (EPI 3; else BN)
+  int nstg;                         // staging buffers per epilogue warp (1 or 2)
 };
 
 constexpr int AG_WARPS = 4, AG_THREADS = AG_WARPS * 32, KOFF_MAX = 2048;
 constexpr int SMEM_AG_BYTES = STAGES * STAGE_BYTES + 1024 + 256 + KOFF_MAX * 8;
+constexpr size_t SMEM_LIMIT = 232448;          // 227 KB per CTA (static + dynamic)
 
 __device__ __forceinline__ void cp_async16(uint32_t dst, const void* src) {
   asm volatile("cp.async.cg.shared.global [%0], [%1], 16;" ::"r"(dst), "l"(src) : "memory");
@@ -218,6 +222,34 @@ __device__ __forceinline__ void mma_commit(uint32_t bar) {
 __device__ __forceinline__ void tc_fence_before() { asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory"); }
 __device__ __forceinline__ void tc_fence_after() { asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory"); }
 
+__device__ __forceinline__ void tmem_ld8(uint32_t taddr, uint32_t* r) {
+  asm volatile("tcgen05.ld.sync.aligned.32x32b.x8.b32 {%0,%1,%2,%3,%4,%5,%6,%7}, [%8];"
+               : "=r"(r[0]), "=r"(r[1]), "=r"(r[2]), "=r"(r[3]), "=r"(r[4]), "=r"(r[5]), "=r"(r[6]), "=r"(r[7])
+               : "r"(taddr));
+}
+__device__ __forceinline__ void tmem_wait_ld() { asm volatile("tcgen05.wait::ld.sync.aligned;" ::: "memory"); }
+__device__ __forceinline__ void bulk_store(void* gdst, uint32_t ssrc, uint32_t bytes, uint64_t pol) {
+  asm volatile("cp.async.bulk.global.shared::cta.bulk_group.L2::cache_hint [%0], [%1], %2, %3;" ::"l"(gdst), "r"(ssrc),
+               "r"(bytes), "l"(pol)
+               : "memory");
+}
+__device__ __forceinline__ uint64_t policy_evict_first() {
+  uint64_t p;
+  asm volatile("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(p));
+  return p;
+}
+__device__ __forceinline__ uint64_t policy_evict_last() {
+  uint64_t p;
+  asm volatile("createpolicy.fractional.L2::evict_last.b64 %0, 1.0;" : "=l"(p));
+  return p;
+}
+__device__ __forceinline__ void tma_load_2d_hint(uint32_t dst, const CUtensorMap* map, uint32_t bar, int c0, int c1,
+                                                 uint64_t pol) {
+  asm volatile(
+      "cp.async.bulk.tensor.2d.shared::cluster.global.mbarrier::complete_tx::bytes.L2::cache_hint [%0], [%1, {%3, %4}], [%2], %5;" ::"r"(dst),
+      "l"((uint64_t)map), "r"(bar), "r"(c0), "r"(c1), "l"(pol)
+      : "memory");
+}
 __device__ __forceinline__ void tmem_ld32(uint32_t taddr, uint32_t* r) {
   asm volatile(
       "tcgen05.ld.sync.aligned.32x32b.x32.b32 "
@@ -237,21 +269,27 @@ __global__ void __launch_bounds__(AG ? THREADS + AG_THREADS : THREADS, 1)
                 const __grid_constant__ Params P) {
   extern __shared__ __align__(1024) uint8_t smem_raw[];
   __shared__ int64_t s_cn[BN];      // column offsets of the current N-tile (scatter epilogue)
+  // ring: NST stages of A (16 KB) and B (bn·128 B); EPI 3 keeps 2 stages to leave room for
+  // the epilogue's staging buffers (K is short where it is used: CCSD(T) K = 72)
+  constexpr int NST = EPI == 3 ? 2 : STAGES;
+  const int bn = EPI == 3 ? P.bn : BN;
+  const uint32_t b_stage = EPI == 3 ? (uint32_t)P.bn * 128u : (uint32_t)B_BYTES;
+  const uint32_t ring = NST * (A_BYTES + b_stage);
   uint8_t* smem = (uint8_t*)(((uintptr_t)smem_raw + 1023) & ~(uintptr_t)1023);
   uint8_t* sA = smem;
-  uint8_t* sB = smem + STAGES * A_BYTES;
-  uint64_t* bars = (uint64_t*)(smem + STAGES * STAGE_BYTES);
-  // bars: full[STAGES], empty[STAGES], tmem_full[2], tmem_empty[2]; then the TMEM slot
-  uint32_t* tmem_slot = (uint32_t*)(bars + 2 * STAGES + 4);
-  int64_t* s_koff = (int64_t*)(smem + STAGES * STAGE_BYTES + 256);    // AG: K-chunk offsets
+  uint8_t* sB = smem + NST * A_BYTES;
+  uint64_t* bars = (uint64_t*)(smem + ring);
+  // bars: full[NST], empty[NST], tmem_full[2], tmem_empty[2]; then the TMEM slot
+  uint32_t* tmem_slot = (uint32_t*)(bars + 2 * NST + 4);
+  int64_t* s_koff = (int64_t*)(smem + ring + 256);    // AG: K-chunk offsets
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
-  const uint32_t full0 = smem_u32(bars), empty0 = smem_u32(bars + STAGES);
-  const uint32_t tfull0 = smem_u32(bars + 2 * STAGES), tempty0 = smem_u32(bars + 2 * STAGES + 2);
+  const uint32_t full0 = smem_u32(bars), empty0 = smem_u32(bars + NST);
+  const uint32_t tfull0 = smem_u32(bars + 2 * NST), tempty0 = smem_u32(bars + 2 * NST + 2);
 
   if (warp == 0 && lane == 0) {
     asm volatile("prefetch.tensormap [%0];" ::"l"((uint64_t)&mapA) : "memory");
     asm volatile("prefetch.tensormap [%0];" ::"l"((uint64_t)&mapB) : "memory");
-    for (int s = 0; s < STAGES; ++s) {
+    for (int s = 0; s < NST; ++s) {
       mbar_init(full0 + 8 * s, AG ? 1 + AG_THREADS : 1);    // AG: TMA(B) + every gather thread
       mbar_init(empty0 + 8 * s, 1);
     }
@@ -274,17 +312,18 @@ __global__ void __launch_bounds__(AG ? THREADS + AG_THREADS : THREADS, 1)
   if (warp == 0) {
     if (lane == 0) {
       // ===== TMA producer =====
+      const uint64_t pol = policy_evict_last();
       int stage = 0;
       uint32_t phase = 0;
       for (int u = u_first(P); u < u_last(P); u += u_step(P)) {
         int mb, nb, kb0, kb1, slot;
         u_decode(P, u, &mb, &nb, &kb0, &kb1, &slot);
-        const int m0 = mb * BM, n0 = nb * BN;
+        const int m0 = mb * BM, n0 = nb * bn;
         for (int kb = kb0; kb < kb1; ++kb) {
           mbar_wait(empty0 + 8 * stage, phase ^ 1);
           const uint32_t fb = full0 + 8 * stage;
-          mbar_expect_tx(fb, AG ? B_BYTES : STAGE_BYTES);
-          const uint32_t a_dst = smem_u32(sA + stage * A_BYTES), b_dst = smem_u32(sB + stage * B_BYTES);
+          mbar_expect_tx(fb, AG ? b_stage : A_BYTES + b_stage);
+          const uint32_t a_dst = smem_u32(sA + stage * A_BYTES), b_dst = smem_u32(sB + stage * b_stage);
           const int k0 = kb * BK;
           if (AG) {
             // A arrives from the gather warps
@@ -292,19 +331,28 @@ __global__ void __launch_bounds__(AG ? THREADS + AG_THREADS : THREADS, 1)
             int cr[5];
             box_coords(P.abox, m0, k0, cr);
             tma_load_nd(a_dst, &mapA, fb, P.abox.rank, cr);
+          } else if (EPI == 3) {       // operands stay in L2 (evict_last) under the output stream
+            if (P.a_mn_major) {
+              tma_load_2d_hint(a_dst, &mapA, fb, m0, k0, pol);
+              tma_load_2d_hint(a_dst + 8192, &mapA, fb, m0 + 64, k0, pol);
+            } else {
+              tma_load_2d_hint(a_dst, &mapA, fb, k0, m0, pol);
+            }
           } else if (P.a_mn_major) {   // box {64 m, 64 k}, two atoms along M
             tma_load_2d(a_dst, &mapA, fb, m0, k0);
             tma_load_2d(a_dst + 8192, &mapA, fb, m0 + 64, k0);
           } else {                     // box {64 k, 128 m}
             tma_load_2d(a_dst, &mapA, fb, k0, m0);
           }
-          if (P.b_mn_major) {          // box {64 n, 64 k}, four atoms along N
+          if (EPI == 3) {              // K-major B, box {64 k, bn n}
+            tma_load_2d_hint(b_dst, &mapB, fb, k0, n0, pol);
+          } else if (P.b_mn_major) {   // box {64 n, 64 k}, four atoms along N
 #pragma unroll
             for (int j = 0; j < 4; ++j) tma_load_2d(b_dst + 8192 * j, &mapB, fb, n0 + 64 * j, k0);
           } else {                     // box {64 k, 256 n}
             tma_load_2d(b_dst, &mapB, fb, k0, n0);
           }
-          if (++stage == STAGES) { stage = 0; phase ^= 1; }
+          if (++stage == NST) { stage = 0; phase ^= 1; }
         }
       }
     }
@@ -324,7 +372,7 @@ __global__ void __launch_bounds__(AG ? THREADS + AG_THREADS : THREADS, 1)
         for (int kb = kb0; kb < kb1; ++kb) {
           mbar_wait(full0 + 8 * stage, phase);
           tc_fence_after();
-          const uint32_t a0 = smem_u32(sA + stage * A_BYTES), b0 = smem_u32(sB + stage * B_BYTES);
+          const uint32_t a0 = smem_u32(sA + stage * A_BYTES), b0 = smem_u32(sB + stage * b_stage);
 #pragma unroll
           for (int k = 0; k < BK / 16; ++k) {
             // K-major: +32 B per 16-element K step inside the 128-B swizzled row;
@@ -334,7 +382,7 @@ __global__ void __launch_bounds__(AG ? THREADS + AG_THREADS : THREADS, 1)
             mma_bf16(d, ad, bd, P.idesc, kb != kb0 || k != 0);
           }
           mma_commit(empty0 + 8 * stage);            // smem stage free once these MMAs retire
-          if (++stage == STAGES) { stage = 0; phase ^= 1; }
+          if (++stage == NST) { stage = 0; phase ^= 1; }
         }
         mma_commit(tfull0 + 8 * acc);                 // accumulator ready for the epilogue
       }
@@ -380,14 +428,104 @@ __global__ void __launch_bounds__(AG ? THREADS + AG_THREADS : THREADS, 1)
           else if (P.ag_lag == 2) cp_async_wait<2>();
           else cp_async_wait<3>();
           fence_proxy_async();
-          mbar_arrive(full0 + 8 * ((g - P.ag_lag) % STAGES));
+          mbar_arrive(full0 + 8 * ((g - P.ag_lag) % NST));
         }
-        if (++stage == STAGES) { stage = 0; phase ^= 1; }
+        if (++stage == NST) { stage = 0; phase ^= 1; }
       }
     }
     cp_async_wait<0>();
     fence_proxy_async();
-    for (int j = g - P.ag_lag < 0 ? 0 : g - P.ag_lag; j < g; ++j) mbar_arrive(full0 + 8 * (j % STAGES));
+    for (int j = g - P.ag_lag < 0 ? 0 : g - P.ag_lag; j < g; ++j) mbar_arrive(full0 + 8 * (j % NST));
+  } else if (EPI == 3) {
+    // ===== bulk-run epilogue: the output is contiguous along n in runs of L = bn/2 and a
+    // warp owns 32 accumulator rows × one run.  TMEM → registers → this warp's staging
+    // buffer in output order [row][L]; then the rows whose offsets continue each other
+    // (cM[m+1] = cM[m] + L, e.g. CCSD(T)'s p5) leave as ONE cp.async.bulk store of
+    // rows·L·4 bytes (measured 6.8-7.2 TB/s for 36-72 KB pieces vs 4.1-5.1 TB/s for
+    // per-thread stores of the same layout, tools/wbw_probe.cu).  Double-buffered
+    // staging: a buffer is rewritten only after its previous bulk read completed. =====
+    const int quad = warp & 3;
+    const int half = (warp - 2) >> 2;
+    const int L = bn >> 1;
+    const int row = quad * 32 + lane;
+    float* stg0 = (float*)(smem + ring + 1024) + (size_t)(warp - 2) * P.nstg * 32 * L;
+    int it = 0, sb = 0;
+    int cached_nb = -1;
+    const uint64_t pol = policy_evict_first();
+    // the row offset cM[m] of the NEXT tile is loaded one iteration ahead (its L2 latency
+    // was the epilogue's largest stall)
+    auto row_off = [&](int u) -> int64_t {
+      if (u >= u_last(P)) return -1;
+      int mb, nbk, kb0, kb1, slot;
+      u_decode(P, u, &mb, &nbk, &kb0, &kb1, &slot);
+      const int64_t m = (int64_t)mb * BM + row;
+      return m < P.M ? P.cbase + __ldg(P.cM + m) : -1;
+    };
+    int64_t crow_next = row_off(u_first(P));
+    for (int u = u_first(P); u < u_last(P); u += u_step(P), ++it) {
+      const int acc = it & 1;
+      int mb, nbk, kb0, kb1, slot;
+      u_decode(P, u, &mb, &nbk, &kb0, &kb1, &slot);
+      const int64_t crow_cur = crow_next;
+      crow_next = row_off(u + u_step(P));
+      if (nbk != cached_nb) {
+        const int et = threadIdx.x - 64;
+        named_sync(1, 256);
+        const int64_t nn = (int64_t)nbk * bn + et;
+        if (et < bn) s_cn[et] = __ldg(P.cN + min(nn, P.N - 1));
+        named_sync(1, 256);
+        cached_nb = nbk;
+      }
+      const bool mok = crow_cur >= 0;
+      const int64_t crow = mok ? crow_cur : 0;
+      const bool nok = (int64_t)nbk * bn + half * L < P.N;
+      float* stg = stg0 + sb * 32 * L;
+      if (lane == 0) {
+        if (P.nstg == 2) asm volatile("cp.async.bulk.wait_group.read 1;" ::: "memory");
+        else asm volatile("cp.async.bulk.wait_group.read 0;" ::: "memory");
+      }
+      __syncwarp();
+      mbar_wait(tfull0 + 8 * acc, (it >> 1) & 1);
+      tc_fence_after();
+      const uint32_t tbase = tmem + ((uint32_t)(quad * 32) << 16) + acc * BN + half * L;
+      float* srow = stg + lane * L;
+#pragma unroll 1
+      for (int c = 0; c < L; c += 16) {
+        uint32_t r[16];
+        tmem_ld8(tbase + c, r);
+        if (c + 8 < L) tmem_ld8(tbase + c + 8, r + 8);
+        tmem_wait_ld();
+        const int nv = c + 8 < L ? 4 : 2;
+#pragma unroll
+        for (int q = 0; q < 4; ++q)
+          if (q < nv)
+            asm volatile("st.shared.v4.b32 [%0], {%1, %2, %3, %4};" ::"r"(smem_u32(srow + c + 4 * q)), "r"(r[4 * q]),
+                         "r"(r[4 * q + 1]), "r"(r[4 * q + 2]), "r"(r[4 * q + 3])
+                         : "memory");
+      }
+      tc_fence_before();
+      mbar_arrive(tempty0 + 8 * acc);          // accumulator free for the MMA of tile it+2
+      fence_proxy_async();
+      __syncwarp();
+      // row pieces: a piece starts where the output offset does not continue the previous row
+      const int64_t prev = __shfl_up_sync(0xffffffffu, crow, 1);
+      const bool start = mok && (lane == 0 || crow != prev + L);
+      unsigned st = __ballot_sync(0xffffffffu, start);
+      const int nvalid = __popc(__ballot_sync(0xffffffffu, mok));
+      if (!nok) st = 0;
+      const int64_t coff = s_cn[half * L];
+      while (st) {
+        const int s0 = __ffs(st) - 1;
+        st &= st - 1;
+        const int e0 = st ? __ffs(st) - 1 : nvalid;
+        const int64_t cs = __shfl_sync(0xffffffffu, crow, s0);
+        if (lane == 0) bulk_store(P.C + cs + coff, smem_u32(stg + s0 * L), (uint32_t)((e0 - s0) * L * 4), pol);
+      }
+      if (lane == 0) asm volatile("cp.async.bulk.commit_group;" ::: "memory");
+      if (P.nstg == 2) sb ^= 1;
+    }
+    if (lane == 0) asm volatile("cp.async.bulk.wait_group 0;" ::: "memory");
+    __syncwarp();
   } else {
     // ===== epilogue: warps 2..9; warp → TMEM lane quadrant (warp % 4) and a half of the
     // 256 accumulator columns (two warps per sub-partition hide the store latency) =====
@@ -402,7 +540,7 @@ __global__ void __launch_bounds__(AG ? THREADS + AG_THREADS : THREADS, 1)
       u_decode(P, u, &mb, &nbk, &kb0, &kb1, &slot);
       const int64_t m = (int64_t)mb * BM + row;
       const int64_t n0 = (int64_t)nbk * BN + half * (BN / 2);
-      if (EPI == 1 && nbk != cached_nb) {
+      if (EPI >= 1 && nbk != cached_nb) {
         // (re)load this N-tile's column offsets into shared memory (epilogue warps only)
         const int et = threadIdx.x - 64;
         named_sync(1, 256);
@@ -468,6 +606,34 @@ __global__ void __launch_bounds__(AG ? THREADS + AG_THREADS : THREADS, 1)
 #pragma unroll
             for (int j = 0; j < 32; ++j)
               if (nb + j < P.N) P.C[crow + nb + j] = __uint_as_float(r[j]);
+          }
+        } else if (EPI == 2) {
+          // run-8 scatter: the output is contiguous along n in aligned runs of 8 (the plan
+          // checked cN and the alignment), so each thread stores its row's 32 columns as
+          // four 32-byte vectors (STG.256; 16 B for bf16) at crow + cN[run start]
+          if (mok) {
+#pragma unroll
+            for (int j = 0; j < 4; ++j) {
+              if (nb + 8 * j < P.N) {
+                const int64_t o = crow + s_cn[half * (BN / 2) + c * 32 + 8 * j];
+                const uint32_t* v = r + 8 * j;
+                if (OUT_BF16) {
+                  uint32_t h[4];
+#pragma unroll
+                  for (int q = 0; q < 4; ++q) {
+                    const __nv_bfloat162 t = __floats2bfloat162_rn(__uint_as_float(v[2 * q]), __uint_as_float(v[2 * q + 1]));
+                    h[q] = *reinterpret_cast<const uint32_t*>(&t);
+                  }
+                  asm volatile("st.global.cs.v4.b32 [%0], {%1, %2, %3, %4};" ::"l"((__nv_bfloat16*)P.C + o), "r"(h[0]),
+                               "r"(h[1]), "r"(h[2]), "r"(h[3])
+                               : "memory");
+                } else {
+                  asm volatile("st.global.cs.v8.b32 [%0], {%1, %2, %3, %4, %5, %6, %7, %8};" ::"l"(P.C + o), "r"(v[0]),
+                               "r"(v[1]), "r"(v[2]), "r"(v[3]), "r"(v[4]), "r"(v[5]), "r"(v[6]), "r"(v[7])
+                               : "memory");
+                }
+              }
+            }
           }
         } else {
           // scatter through the output tables: column offsets first (branch-free,
@@ -967,6 +1133,8 @@ struct T4State {
   t4::Params P;
   int cg = 1;      // 1: one SM per 128×256 tile; 2: SM pair per 256×256 tile
   bool ag = false; // A staged by the kernel's gather warps (no A tensor map, no pre-pass)
+  int epi = 1;      // 0 row-major C, 1 per-element scatter, 2 run-8 vector scatter, 3 bulk runs
+  size_t smem3 = 0; // dynamic shared memory of the EPI 3 kernel
   int tail_parts = 0;   // 1-SM split-K tail: partial tiles in the workspace at tail_off
   int grid1 = 0;        // its grid (the SM count at plan time: one tail unit per CTA)
   size_t tail_off = 0;
@@ -1107,6 +1275,20 @@ mdh_status prepare_t4(Plan* p) {
   P.ldc = sm;
   P.cbase = p->out[0].acc[0].base;
   P.sched = P.c_rowmajor ? 0 : 1;
+  // run-8 scatter epilogue (EPI 2): cN in aligned runs of 8 consecutive elements and every
+  // row offset a multiple of 8, so a thread's 8 consecutive accumulators are one vector
+  s->epi = P.c_rowmajor ? 0 : 1;
+  if (!P.c_rowmajor && c.N % 8 == 0) {
+    bool run8 = true;
+    for (size_t i = 0; i < cn.size() && run8; i += 8) {
+      if ((P.cbase + cn[i]) % 8) run8 = false;
+      for (int j = 1; j < 8 && run8; ++j)
+        if (cn[i + j] != cn[i] + j) run8 = false;
+    }
+    for (size_t i = 0; i < cm.size() && run8; ++i)
+      if (cm[i] % 8) run8 = false;
+    if (run8) s->epi = 2;
+  }
   // 2-SM pairs (cta_group::2, 256×256 tiles) for large row-major outputs (measured 1290 vs
   // 1170 TFLOP/s on MatMul 4096³); tile knob cluster=1 forces the 1-SM kernel
   // (the in-kernel A gather is a 1-SM kernel: a 2-SM version, whose peer CTA must publish
@@ -1151,14 +1333,49 @@ mdh_status prepare_t4(Plan* p) {
       s->grid1 = C;
     }
   }
+  // bulk-run epilogue (EPI 3): the output is contiguous along n in runs of L elements
+  // (cN[iL + j] = cN[iL] + j), 32 ≤ L ≤ 128, L % 8 == 0, N % L == 0, 16-byte aligned run
+  // starts and row offsets; the N-tile becomes 2L wide so every tile holds whole runs and
+  // a warp's rows go out as contiguous cp.async.bulk stores (CCSD(T): L = 72, bn = 144).
+  // fp32 output, 1-SM kernel, TMA-fed A, K-major B, no split tail; tile knob epi=0 disables.
+  P.bn = t4::BN;
+  P.nstg = 0;
+  if (s->epi != 0 && !P.out_bf16 && s->cg == 1 && !a_gather && !a_box && !s->b.mn_major && s->tail_parts == 0 &&
+      p->tiles.epi != 1) {
+    int64_t L = 1;
+    while (L < c.N && cn[(size_t)L] == cn[0] + L) ++L;
+    bool ok = L >= 32 && L <= 128 && L % 8 == 0 && c.N % L == 0;
+    for (int64_t i = 0; i < c.N && ok; i += L) {
+      if ((P.cbase + cn[(size_t)i]) % 4) ok = false;
+      for (int64_t j = 1; j < L && ok; ++j)
+        if (cn[(size_t)(i + j)] != cn[(size_t)i] + j) ok = false;
+    }
+    for (size_t i = 0; i < cm.size() && ok; ++i)
+      if (cm[i] % 4) ok = false;
+    if (ok) {
+      const int bn = (int)(2 * L);
+      const size_t ring = 2 * ((size_t)t4::A_BYTES + (size_t)bn * 128);
+      const size_t stg1 = (size_t)8 * 32 * L * 4;
+      const size_t lim = t4::SMEM_LIMIT - 1024 - t4::BN * sizeof(int64_t);
+      P.nstg = ring + 1024 + 2 * stg1 <= lim ? 2 : (ring + 1024 + stg1 <= lim ? 1 : 0);
+      if (P.nstg > 0) {
+        s->epi = 3;
+        P.bn = bn;
+        P.tiles_n = (int)((c.N + bn - 1) / bn);
+        P.num_tiles = P.tiles_m * P.tiles_n;
+        P.idesc = (P.idesc & ~(0x3Fu << 17)) | ((uint32_t)(bn >> 3) << 17);
+        s->smem3 = ring + 1024 + P.nstg * stg1 + 1024;
+      }
+    }
+  }
   p->tmaps = s;
   p->t4_variant = 1 + (s->a.permuted ? 2 : 0) + (s->b.permuted ? 4 : 0) + (s->cg == 2 ? 8 : 0) + (a_box ? 16 : 0) +
-                  (a_gather ? 32 : 0);
+                  (a_gather ? 32 : 0) + (s->epi == 2 ? 64 : 0) + (s->epi == 3 ? 128 : 0);
   p->ws_kernel = ws;
   p->tiles.bm = s->cg == 2 ? 256 : t4::BM;
-  p->tiles.bn = t4::BN;
+  p->tiles.bn = s->epi == 3 ? P.bn : t4::BN;
   p->tiles.bk = t4::BK;
-  p->tiles.stages = s->cg == 2 ? t4::S2 : t4::STAGES;
+  p->tiles.stages = s->cg == 2 ? t4::S2 : (s->epi == 3 ? 2 : t4::STAGES);
   p->tiles.cluster = s->cg;
   return MDH_OK;
 }
@@ -1271,21 +1488,28 @@ mdh_status launch_t4(const Plan& p, const void* const* in, void* const* out, voi
   } else if (s->a.mn_major) MDH_TRY(make_map(&ma, A, c.M, c.K, s->a.ld, 64, 64));
   else MDH_TRY(make_map(&ma, A, c.K, c.M, s->a.ld, 64, 128));
   if (s->b.mn_major) MDH_TRY(make_map(&mb, B, c.N, c.K, s->b.ld, 64, 64));
-  else MDH_TRY(make_map(&mb, B, c.K, c.N, s->b.ld, 64, s->cg == 2 ? 128 : 256));
+  else MDH_TRY(make_map(&mb, B, c.K, c.N, s->b.ld, 64, s->cg == 2 ? 128 : (uint32_t)P.bn));
   if (s->ag) ma = mb;
   static std::once_flag attr_once;
   static cudaError_t attr_err = cudaSuccess;
   std::call_once(attr_once, [] {
-    const void* ks[3] = {(const void*)t4::gemm_kernel<0, false>, (const void*)t4::gemm_kernel<1, false>,
-                         (const void*)t4::gemm_kernel<1, true>};
+    const void* ks[5] = {(const void*)t4::gemm_kernel<0, false>, (const void*)t4::gemm_kernel<1, false>,
+                         (const void*)t4::gemm_kernel<1, true>, (const void*)t4::gemm_kernel<2, false>,
+                         (const void*)t4::gemm_kernel<2, true>};
     for (const void* k : ks) {
       cudaError_t e = cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, t4::SMEM_BYTES);
       if (e != cudaSuccess) attr_err = e;
     }
-    const void* kg[3] = {(const void*)t4::gemm_kernel<0, false, true>, (const void*)t4::gemm_kernel<1, false, true>,
-                         (const void*)t4::gemm_kernel<1, true, true>};
+    const void* kg[5] = {(const void*)t4::gemm_kernel<0, false, true>, (const void*)t4::gemm_kernel<1, false, true>,
+                         (const void*)t4::gemm_kernel<1, true, true>, (const void*)t4::gemm_kernel<2, false, true>,
+                         (const void*)t4::gemm_kernel<2, true, true>};
     for (const void* k : kg) {
       cudaError_t e = cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, t4::SMEM_AG_BYTES);
+      if (e != cudaSuccess) attr_err = e;
+    }
+    {
+      cudaError_t e = cudaFuncSetAttribute((const void*)t4::gemm_kernel<3, false>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                           (int)(t4::SMEM_LIMIT - t4::BN * sizeof(int64_t)));
       if (e != cudaSuccess) attr_err = e;
     }
     const void* k2[2] = {(const void*)t4::gemm2_kernel<true>, (const void*)t4::gemm2_kernel<false>};
@@ -1329,15 +1553,29 @@ mdh_status launch_t4(const Plan& p, const void* const* in, void* const* out, voi
     P.part = (float*)((char*)ws + s->tail_off);
     P.tail_cnt = (unsigned*)((char*)ws + s->tail_off + (size_t)s->tail_parts * t4::BM * t4::BN * sizeof(float));
   }
+  // EPI 2 needs a 32-byte (fp32) / 16-byte (bf16) aligned output base
+  const bool epi2 = s->epi == 2 && (uintptr_t)P.C % (P.out_bf16 ? 16 : 32) == 0;
   if (s->ag) {
     P.ag_lag = 2;   // measured on MCC conv5_1: lag 1 / 2 / 3 → 89 / 83 / 130 µs
     constexpr int TG = t4::THREADS + t4::AG_THREADS;
     if (P.c_rowmajor && !P.out_bf16) t4::gemm_kernel<0, false, true><<<grid, TG, t4::SMEM_AG_BYTES, st>>>(ma, mb, P);
+    else if (epi2 && !P.out_bf16) t4::gemm_kernel<2, false, true><<<grid, TG, t4::SMEM_AG_BYTES, st>>>(ma, mb, P);
+    else if (epi2) t4::gemm_kernel<2, true, true><<<grid, TG, t4::SMEM_AG_BYTES, st>>>(ma, mb, P);
     else if (!P.out_bf16) t4::gemm_kernel<1, false, true><<<grid, TG, t4::SMEM_AG_BYTES, st>>>(ma, mb, P);
     else t4::gemm_kernel<1, true, true><<<grid, TG, t4::SMEM_AG_BYTES, st>>>(ma, mb, P);
     return post_launch("t4_gemm_kernel_ag");
   }
+  if (s->epi == 3 && (uintptr_t)P.C % 16 == 0) {
+    t4::gemm_kernel<3, false><<<grid, t4::THREADS, s->smem3, st>>>(ma, mb, P);
+    return post_launch("t4_gemm_kernel_bulk");
+  }
+  if (s->epi == 3) {          // unaligned output base: the per-element scatter with 256-wide tiles
+    set_error("T4 bulk-run epilogue: output base not 16-byte aligned");
+    return MDH_ERR_INVALID_ARG;
+  }
   if (P.c_rowmajor && !P.out_bf16) t4::gemm_kernel<0, false><<<grid, t4::THREADS, t4::SMEM_BYTES, st>>>(ma, mb, P);
+  else if (epi2 && !P.out_bf16) t4::gemm_kernel<2, false><<<grid, t4::THREADS, t4::SMEM_BYTES, st>>>(ma, mb, P);
+  else if (epi2) t4::gemm_kernel<2, true><<<grid, t4::THREADS, t4::SMEM_BYTES, st>>>(ma, mb, P);
   else if (!P.out_bf16) t4::gemm_kernel<1, false><<<grid, t4::THREADS, t4::SMEM_BYTES, st>>>(ma, mb, P);
   else t4::gemm_kernel<1, true><<<grid, t4::THREADS, t4::SMEM_BYTES, st>>>(ma, mb, P);
   return post_launch("t4_gemm_kernel");

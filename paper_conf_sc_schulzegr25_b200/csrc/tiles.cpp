@@ -144,6 +144,7 @@ void apply(Tiles* t, const std::string& k, double v) {
   else if (k == "per_thread") t->per_thread = iv;
   else if (k == "cluster") t->cluster = iv;
   else if (k == "implicit") t->implicit = iv;
+  else if (k == "epi") t->epi = iv;
 }
 
 std::string read_file(const char* path) {

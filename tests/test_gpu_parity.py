@@ -447,3 +447,25 @@ def test_mcc_bf16_config_sampled():
     x = G.mcc_inputs(spec)
     got, _ = run_gpu(spec, x)
     assert_close_points(spec, x, got, 1e-2, n=5000, kind="scale")
+
+
+@pytest.mark.parametrize("case", ["bulk_ragged", "bulk_O4_V72", "run8_sd2", "run8_forced"])
+def test_t4_scatter_epilogues(case):
+    """T4 scatter epilogues on CCSD(T)-shaped outputs (orientation swapped so t3's unit-stride
+    p4 is on the TMEM column axis): EPI 3 bulk runs (L = V, N-tile 2L; ragged M, a last
+    N-tile holding one run, row pieces broken at h3 and tile edges), EPI 2 run-8 vectors
+    (sd2: p4 runs of 16; sd1 with the bulk kernel disabled by tile knob epi=1)."""
+    spec, tile, bit = {
+        "bulk_ragged": (S.ccsd_sd1(3, 40, "bf16"), None, 128),
+        "bulk_O4_V72": (S.ccsd_sd1(4, 72, "bf16"), None, 128),
+        "run8_sd2": (S.ccsd_sd2(dtype="bf16"), None, 64),
+        "run8_forced": (S.ccsd_sd1(3, 40, "bf16"), "epi=1", 64),
+    }[case]
+    x = G.gen_inputs(spec, 4020)
+    got, p = run_gpu(spec, x, force_tile=tile)
+    v = p.describe()["t4_variant"]
+    assert v & bit, v
+    if case == "bulk_O4_V72":
+        assert_close_points(spec, x, got, 1e-2, n=50000, kind="scale")
+    else:
+        assert_close_full(spec, x, got, 1e-2, kind="scale")
