@@ -81,11 +81,15 @@ struct Params {
   // bulk-run epilogue (EPI 3): N-tile = 2 output runs of bn/2 contiguous elements
   int bn;                           // N-tile width (EPI 3; else BN)
   int nstg;                         // staging buffers per epilogue warp (1 or 2)
+  int e3flip;                       // EPI 3 bank-conflict-free staging order (tile knob epi=2: off)
+  int bres;                         // EPI 3: B of the current N-tile resident in shared memory
 };
 
 constexpr int AG_WARPS = 4, AG_THREADS = AG_WARPS * 32, KOFF_MAX = 2048;
 constexpr int SMEM_AG_BYTES = STAGES * STAGE_BYTES + 1024 + 256 + KOFF_MAX * 8;
 constexpr size_t SMEM_LIMIT = 232448;          // 227 KB per CTA (static + dynamic)
+constexpr int EPI3_LMAX = 128;                 // longest output run the bulk-run epilogue takes
+
 
 __device__ __forceinline__ void cp_async16(uint32_t dst, const void* src) {
   asm volatile("cp.async.cg.shared.global [%0], [%1], 16;" ::"r"(dst), "l"(src) : "memory");
@@ -274,17 +278,22 @@ __global__ void __launch_bounds__(AG ? THREADS + AG_THREADS : THREADS, 1)
   constexpr int NST = EPI == 3 ? 2 : STAGES;
   const int bn = EPI == 3 ? P.bn : BN;
   const uint32_t b_stage = EPI == 3 ? (uint32_t)P.bn * 128u : (uint32_t)B_BYTES;
-  const uint32_t ring = NST * (A_BYTES + b_stage);
+  // B-resident mode (EPI 3, P.bres): the whole K extent of the current N-tile's B stays in
+  // shared memory while the CTA walks its M-tiles (sched 1 keeps one N-tile for hundreds of
+  // consecutive tiles), so only A streams through the ring
+  const bool bres = EPI == 3 && P.bres;
+  const uint32_t ring = bres ? NST * A_BYTES + P.num_kb * b_stage : NST * (A_BYTES + b_stage);
   uint8_t* smem = (uint8_t*)(((uintptr_t)smem_raw + 1023) & ~(uintptr_t)1023);
   uint8_t* sA = smem;
   uint8_t* sB = smem + NST * A_BYTES;
   uint64_t* bars = (uint64_t*)(smem + ring);
-  // bars: full[NST], empty[NST], tmem_full[2], tmem_empty[2]; then the TMEM slot
-  uint32_t* tmem_slot = (uint32_t*)(bars + 2 * NST + 4);
+  // bars: full[NST], empty[NST], tmem_full[2], tmem_empty[2], b_full, b_empty; then the TMEM slot
+  uint32_t* tmem_slot = (uint32_t*)(bars + 2 * NST + 6);
   int64_t* s_koff = (int64_t*)(smem + ring + 256);    // AG: K-chunk offsets
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const uint32_t full0 = smem_u32(bars), empty0 = smem_u32(bars + NST);
   const uint32_t tfull0 = smem_u32(bars + 2 * NST), tempty0 = smem_u32(bars + 2 * NST + 2);
+  const uint32_t bfull = smem_u32(bars + 2 * NST + 4), bempty = smem_u32(bars + 2 * NST + 5);
 
   if (warp == 0 && lane == 0) {
     asm volatile("prefetch.tensormap [%0];" ::"l"((uint64_t)&mapA) : "memory");
@@ -297,6 +306,8 @@ __global__ void __launch_bounds__(AG ? THREADS + AG_THREADS : THREADS, 1)
       mbar_init(tfull0 + 8 * a, 1);
       mbar_init(tempty0 + 8 * a, 256);
     }
+    mbar_init(bfull, 1);
+    mbar_init(bempty, 1);
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
   }
   if (warp == 1) {
@@ -315,14 +326,23 @@ __global__ void __launch_bounds__(AG ? THREADS + AG_THREADS : THREADS, 1)
       const uint64_t pol = policy_evict_last();
       int stage = 0;
       uint32_t phase = 0;
+      int b_nb = -1, b_loads = 0;
       for (int u = u_first(P); u < u_last(P); u += u_step(P)) {
         int mb, nb, kb0, kb1, slot;
         u_decode(P, u, &mb, &nb, &kb0, &kb1, &slot);
         const int m0 = mb * BM, n0 = nb * bn;
+        if (bres && nb != b_nb) {               // (re)load the resident B of this N-tile
+          if (b_loads > 0) mbar_wait(bempty, (b_loads - 1) & 1);
+          mbar_expect_tx(bfull, (uint32_t)P.num_kb * b_stage);
+          for (int kb = 0; kb < P.num_kb; ++kb)
+            tma_load_2d_hint(smem_u32(sB + kb * b_stage), &mapB, bfull, kb * BK, n0, pol);
+          b_nb = nb;
+          ++b_loads;
+        }
         for (int kb = kb0; kb < kb1; ++kb) {
           mbar_wait(empty0 + 8 * stage, phase ^ 1);
           const uint32_t fb = full0 + 8 * stage;
-          mbar_expect_tx(fb, AG ? b_stage : A_BYTES + b_stage);
+          mbar_expect_tx(fb, AG ? b_stage : (bres ? A_BYTES : A_BYTES + b_stage));
           const uint32_t a_dst = smem_u32(sA + stage * A_BYTES), b_dst = smem_u32(sB + stage * b_stage);
           const int k0 = kb * BK;
           if (AG) {
@@ -344,7 +364,9 @@ __global__ void __launch_bounds__(AG ? THREADS + AG_THREADS : THREADS, 1)
           } else {                     // box {64 k, 128 m}
             tma_load_2d(a_dst, &mapA, fb, k0, m0);
           }
-          if (EPI == 3) {              // K-major B, box {64 k, bn n}
+          if (bres) {
+            // B is resident
+          } else if (EPI == 3) {       // K-major B, box {64 k, bn n}
             tma_load_2d_hint(b_dst, &mapB, fb, k0, n0, pol);
           } else if (P.b_mn_major) {   // box {64 n, 64 k}, four atoms along N
 #pragma unroll
@@ -362,17 +384,25 @@ __global__ void __launch_bounds__(AG ? THREADS + AG_THREADS : THREADS, 1)
       int stage = 0;
       uint32_t phase = 0;
       int it = 0;
+      int b_nb = -1, b_uses = 0;
       for (int u = u_first(P); u < u_last(P); u += u_step(P), ++it) {
         int mb, nb, kb0, kb1, slot;
         u_decode(P, u, &mb, &nb, &kb0, &kb1, &slot);
         const int acc = it & 1;
+        if (bres && nb != b_nb) {
+          if (b_uses > 0) mma_commit(bempty);   // the old B is free once the MMAs issued so far retire
+          mbar_wait(bfull, b_uses & 1);
+          b_nb = nb;
+          ++b_uses;
+        }
         mbar_wait(tempty0 + 8 * acc, ((it >> 1) & 1) ^ 1);
         tc_fence_after();
         const uint32_t d = tmem + acc * BN;
         for (int kb = kb0; kb < kb1; ++kb) {
           mbar_wait(full0 + 8 * stage, phase);
           tc_fence_after();
-          const uint32_t a0 = smem_u32(sA + stage * A_BYTES), b0 = smem_u32(sB + stage * b_stage);
+          const uint32_t a0 = smem_u32(sA + stage * A_BYTES),
+                         b0 = smem_u32(sB + (bres ? kb : stage) * b_stage);
 #pragma unroll
           for (int k = 0; k < BK / 16; ++k) {
             // K-major: +32 B per 16-element K step inside the 128-B swizzled row;
@@ -488,20 +518,33 @@ __global__ void __launch_bounds__(AG ? THREADS + AG_THREADS : THREADS, 1)
       mbar_wait(tfull0 + 8 * acc, (it >> 1) & 1);
       tc_fence_after();
       const uint32_t tbase = tmem + ((uint32_t)(quad * 32) << 16) + acc * BN + half * L;
-      float* srow = stg + lane * L;
+      // 16 columns per batch of two x8 loads (one wait), then 16-byte st.shared in pairs of
+      // chunks; lanes with bit 2 set take the pair in the other order, which makes each
+      // 8-lane phase hit 8 distinct bank groups (row pitch L·4 B ≡ 2 groups mod 8 for L = 72)
+      const uint32_t srow = smem_u32(stg + lane * L);
+      const bool flip = P.e3flip && ((lane >> 2) & 1);
 #pragma unroll 1
       for (int c = 0; c < L; c += 16) {
         uint32_t r[16];
         tmem_ld8(tbase + c, r);
         if (c + 8 < L) tmem_ld8(tbase + c + 8, r + 8);
         tmem_wait_ld();
-        const int nv = c + 8 < L ? 4 : 2;
 #pragma unroll
-        for (int q = 0; q < 4; ++q)
-          if (q < nv)
-            asm volatile("st.shared.v4.b32 [%0], {%1, %2, %3, %4};" ::"r"(smem_u32(srow + c + 4 * q)), "r"(r[4 * q]),
-                         "r"(r[4 * q + 1]), "r"(r[4 * q + 2]), "r"(r[4 * q + 3])
+        for (int h = 0; h < 16; h += 8) {
+          if (c + h < L) {
+            uint32_t v[8];
+#pragma unroll
+            for (int j = 0; j < 4; ++j) {
+              v[j] = flip ? r[h + 4 + j] : r[h + j];
+              v[4 + j] = flip ? r[h + j] : r[h + 4 + j];
+            }
+            const uint32_t a0 = srow + 4 * (c + h + (flip ? 4 : 0)), a1 = srow + 4 * (c + h + (flip ? 0 : 4));
+            asm volatile("st.shared.v4.b32 [%0], {%1, %2, %3, %4};" ::"r"(a0), "r"(v[0]), "r"(v[1]), "r"(v[2]), "r"(v[3])
                          : "memory");
+            asm volatile("st.shared.v4.b32 [%0], {%1, %2, %3, %4};" ::"r"(a1), "r"(v[4]), "r"(v[5]), "r"(v[6]), "r"(v[7])
+                         : "memory");
+          }
+        }
       }
       tc_fence_before();
       mbar_arrive(tempty0 + 8 * acc);          // accumulator free for the MMA of tile it+2
@@ -1340,11 +1383,12 @@ mdh_status prepare_t4(Plan* p) {
   // fp32 output, 1-SM kernel, TMA-fed A, K-major B, no split tail; tile knob epi=0 disables.
   P.bn = t4::BN;
   P.nstg = 0;
+  P.e3flip = p->tiles.epi != 2;
   if (s->epi != 0 && !P.out_bf16 && s->cg == 1 && !a_gather && !a_box && !s->b.mn_major && s->tail_parts == 0 &&
       p->tiles.epi != 1) {
     int64_t L = 1;
     while (L < c.N && cn[(size_t)L] == cn[0] + L) ++L;
-    bool ok = L >= 32 && L <= 128 && L % 8 == 0 && c.N % L == 0;
+    bool ok = L >= 32 && L <= t4::EPI3_LMAX && L % 8 == 0 && c.N % L == 0;
     for (int64_t i = 0; i < c.N && ok; i += L) {
       if ((P.cbase + cn[(size_t)i]) % 4) ok = false;
       for (int64_t j = 1; j < L && ok; ++j)
@@ -1354,9 +1398,12 @@ mdh_status prepare_t4(Plan* p) {
       if (cm[i] % 4) ok = false;
     if (ok) {
       const int bn = (int)(2 * L);
-      const size_t ring = 2 * ((size_t)t4::A_BYTES + (size_t)bn * 128);
       const size_t stg1 = (size_t)8 * 32 * L * 4;
       const size_t lim = t4::SMEM_LIMIT - 1024 - t4::BN * sizeof(int64_t);
+      // B resident when its whole K extent fits beside two A stages and double-buffered staging
+      const size_t ring_res = 2 * (size_t)t4::A_BYTES + (size_t)P.num_kb * bn * 128;
+      P.bres = p->tiles.epi != 3 && ring_res + 1024 + 2 * stg1 <= lim;
+      const size_t ring = P.bres ? ring_res : 2 * ((size_t)t4::A_BYTES + (size_t)bn * 128);
       P.nstg = ring + 1024 + 2 * stg1 <= lim ? 2 : (ring + 1024 + stg1 <= lim ? 1 : 0);
       if (P.nstg > 0) {
         s->epi = 3;
