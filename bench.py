@@ -90,6 +90,16 @@ def workload(name, world=1, rank=0):
         spec = S.mcc(256, 7, 7, 512, 3, 3, 512, "bf16")
         return dict(spec=spec, inputs=lambda: G.mcc_inputs(spec), work=2.0 * 256 * 49 * 512 * 4608, unit="TFLOP/s",
                     scale=1e12, bound="tensor", dtype="bf16", desc="MCC ResNet-50 conv5_1 3x3/s2 N=256 bf16")
+    if name == "gaussian2d":
+        I = J = 4096
+        spec = S.gaussian2d(I, J)
+        return dict(spec=spec, inputs=lambda: G.gaussian2d_inputs(I, J), work=4.0 * ((I + 4) * (J + 4) + I * J),
+                    unit="GB/s", scale=1e9, bound="hbm", dtype="f32",
+                    desc="Gaussian_2D 5x5 4096^2 fp32 (Fig 3 P:520-521; reading C-31)")
+    if name == "matvec_4096":
+        spec = S.matvec(4096, 4096)
+        return dict(spec=spec, inputs=lambda: G.gen_inputs(spec, 2100), work=4.0 * (4096 * 4096 + 4096 + 4096),
+                    unit="GB/s", scale=1e9, bound="hbm", dtype="f32", desc="MatVec 4096^2 fp32 (Fig 3 P:514)")
     if name == "prefix_sum_f32":
         spec = S.prefix_sum([1 << 26], 0)
         return dict(spec=spec, inputs=lambda: G.gen_inputs(spec, 6100, "positive"), work=8.0 * (1 << 26),
@@ -108,8 +118,8 @@ def workload(name, world=1, rank=0):
     raise SystemExit(f"unknown workload {name}")
 
 
-SUITE = ["dot_f32", "dot_i32", "dot_f32_2^28", "matvec_f32", "jacobi3d", "matmul_f32", "matmul_bf16",
-         "ccsd_bf16", "mcc_bf16", "prl_A", "prl_B", "prefix_sum_f32", "mbbs_f32"]
+SUITE = ["dot_f32", "dot_i32", "dot_f32_2^28", "matvec_f32", "matvec_4096", "jacobi3d", "gaussian2d", "matmul_f32",
+         "matmul_bf16", "ccsd_bf16", "mcc_bf16", "prl_A", "prl_B", "prefix_sum_f32", "mbbs_f32"]
 
 
 def roofline(w, seconds, pk):

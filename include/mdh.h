@@ -37,11 +37,11 @@
 extern "C" {
 #endif
 
-#define MDH_ABI_VERSION 1
+#define MDH_ABI_VERSION 2  /* 2: MDH_MAX_ACC 8 -> 32 */
 
 #define MDH_MAX_D     10  /* MCC_Caps is 10-D (Fig 3); configs need <= 7        */
 #define MDH_MAX_RANK   8  /* buffer rank                                                */
-#define MDH_MAX_ACC    8  /* accesses per buffer (Jacobi3D: 7 to one buffer) */
+#define MDH_MAX_ACC   32  /* accesses per buffer (Gaussian_2D 5x5: 25 to one image) */
 #define MDH_MAX_BUFS  32  /* PRL: 17 inputs + 3 outputs (Listing 11)         */
 #define MDH_MAX_WORLD 64  /* ranks of one multi-GPU plan                                */
 

@@ -133,6 +133,16 @@ def jacobi3d_inputs(Z, Y, X, kind="random", seed_base=3000):
     return [g.uniform(0.0, 1.0, size=(Z, Y, X)).astype(np.float32)]
 
 
+def gaussian2d_inputs(I, J, kind="random", seed_base=3100):
+    """Gaussian_2D image (I+4)×(J+4) fp32: U[0,1) pixel intensities, or closed-form fields."""
+    if kind == "constant":
+        return [np.full((I + 4, J + 4), 3.0, np.float32)]
+    if kind == "linear":       # x + 2y (exact in fp32 for these sizes)
+        y, x = np.indices((I + 4, J + 4), dtype=np.float32)
+        return [np.ascontiguousarray(x + 2 * y, dtype=np.float32)]
+    return [rng(seed_base + 1).uniform(0.0, 1.0, size=(I + 4, J + 4)).astype(np.float32)]
+
+
 def ccsd_inputs(spec, kind="signed", seed_base=4000):
     return gen_inputs(spec, seed_base, kind)
 

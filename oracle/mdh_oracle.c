@@ -45,7 +45,8 @@
 
 #define O_MAXD 10
 #define O_MAXR 8
-#define O_MAXA 8
+#define O_MAXA 32  /* accesses per buffer (Gaussian_2D: 25 to one image, reading C-31) */
+#define O_MAXX 40  /* input accesses in total (leaf gather array)                     */
 #define O_MAXB 32
 #define O_MAGIC 0x4D44484FLL /* 'MDHO' */
 
@@ -215,8 +216,8 @@ static int64_t wrap(int kind, int64_t v) {
 /* ------------------------------------------------------------ catalog: f (SF) */
 /* Leaf: y(i) = f(x(i)), x gathered through every input access in (b, a) order. */
 static void leaf(const ospec* s, const void* const* in, const int64_t* idx, otuple* y) {
-  double xf[O_MAXB * O_MAXA] = {0};
-  int64_t xi[O_MAXB * O_MAXA] = {0};
+  double xf[O_MAXX] = {0};
+  int64_t xi[O_MAXX] = {0};
   int n = 0;
   for (int b = 0; b < s->nin; ++b) {
     const obuf* B = &s->b[b];
@@ -345,6 +346,7 @@ static int check_catalog(ospec* s, char* err, int cap) {
   }
   int nout_acc = 0;
   for (int b = 0; b < s->nout; ++b) nout_acc += s->b[s->nin + b].nacc;
+  if (nacc > O_MAXX) { seterr(err, cap, "more than 40 input accesses"); return -1; }
   int redop = -1;
   for (int t = 0; t < s->nred; ++t) {
     if (redop >= 0 && s->op[s->red[t]] != redop) { /* reading C-3: evaluated anyway */ }
@@ -385,31 +387,33 @@ static int prepare(const int64_t* enc, int64_t n, const double* fp, int nfp, osp
 /* Shapes (declared or inferred) of all buffers: out[(b)*8 + r]. */
 int mdho_shapes(const int64_t* enc, int64_t n, const double* fp, int nfp, int64_t* shapes,
                 char* err, int cap) {
-  ospec s;
-  if (prepare(enc, n, fp, nfp, &s, err, cap)) return -1;
-  for (int b = 0; b < s.nin + s.nout; ++b)
-    for (int r = 0; r < O_MAXR; ++r) shapes[b * O_MAXR + r] = r < s.b[b].rank ? s.b[b].shape[r] : 0;
-  return 0;
+  ospec* sp = (ospec*)calloc(1, sizeof(ospec));   /* ~0.7 MB: heap, not stack */
+  if (!sp) { seterr(err, cap, "oom"); return -1; }
+  if (prepare(enc, n, fp, nfp, sp, err, cap)) { free(sp); return -1; }
+  for (int b = 0; b < sp->nin + sp->nout; ++b)
+    for (int r = 0; r < O_MAXR; ++r) shapes[b * O_MAXR + r] = r < sp->b[b].rank ? sp->b[b].shape[r] : 0;
+  { free(sp); return 0; }
 }
 
 /* Full evaluation.  Float outputs are written as fp64 arrays; integer outputs in
  * their own type.  Elements outside the image of ω are untouched (reading C-5). */
 int mdho_eval(const int64_t* enc, int64_t n, const double* fp, int nfp,
               const void* const* in, void* const* out, int nthreads, char* err, int cap) {
-  ospec s;
-  if (prepare(enc, n, fp, nfp, &s, err, cap)) return -1;
+  ospec* sp = (ospec*)calloc(1, sizeof(ospec));   /* ~0.7 MB: heap, not stack */
+  if (!sp) { seterr(err, cap, "oom"); return -1; }
+  if (prepare(enc, n, fp, nfp, sp, err, cap)) { free(sp); return -1; }
   unsigned char* mark[O_MAXB];
-  for (int b = 0; b < s.nout; ++b) {
-    mark[b] = (unsigned char*)calloc((size_t)buf_elems(&s.b[s.nin + b]), 1);
-    if (!mark[b]) { seterr(err, cap, "oom"); return -1; }
+  for (int b = 0; b < sp->nout; ++b) {
+    mark[b] = (unsigned char*)calloc((size_t)buf_elems(&sp->b[sp->nin + b]), 1);
+    if (!mark[b]) { seterr(err, cap, "oom"); { free(sp); return -1; } }
   }
   int collide = 0;
-  int64_t outer = s.ncc > 0 ? s.size[s.cc[0]] : 1;
+  int64_t outer = sp->ncc > 0 ? sp->size[sp->cc[0]] : 1;
   int64_t inner = 1;
-  for (int t = 1; t < s.ncc; ++t) inner *= s.size[s.cc[t]];
+  for (int t = 1; t < sp->ncc; ++t) inner *= sp->size[sp->cc[t]];
 #ifdef _OPENMP
   if (nthreads > 0) omp_set_num_threads(nthreads);
-#pragma omp parallel for schedule(dynamic, 1) if (s.ncc > 0)
+#pragma omp parallel for schedule(dynamic, 1) if (sp->ncc > 0)
 #endif
   for (int64_t o = 0; o < outer; ++o) {
     int64_t idx[O_MAXD];
@@ -418,21 +422,21 @@ int mdho_eval(const int64_t* enc, int64_t n, const double* fp, int nfp,
     for (int64_t q = 0; q < inner; ++q) {
       /* cc coordinate j in lexicographic (dimension) order */
       int64_t rem = q;
-      for (int t = s.ncc - 1; t >= 1; --t) {
-        idx[s.cc[t]] = rem % s.size[s.cc[t]];
-        rem /= s.size[s.cc[t]];
+      for (int t = sp->ncc - 1; t >= 1; --t) {
+        idx[sp->cc[t]] = rem % sp->size[sp->cc[t]];
+        rem /= sp->size[sp->cc[t]];
       }
-      if (s.ncc > 0) idx[s.cc[0]] = o;
+      if (sp->ncc > 0) idx[sp->cc[0]] = o;
       memset(&y, 0, sizeof(y));
       int64_t keep[O_MAXD];
       memcpy(keep, idx, sizeof(keep));
-      fold(&s, in, idx, keep, 0, &y);
-      store(&s, out, idx, &y, mark, &collide);
+      fold(sp, in, idx, keep, 0, &y);
+      store(sp, out, idx, &y, mark, &collide);
     }
   }
-  for (int b = 0; b < s.nout; ++b) free(mark[b]);
-  if (collide) { seterr(err, cap, "output index function not injective (reading C-5)"); return -2; }
-  return 0;
+  for (int b = 0; b < sp->nout; ++b) free(mark[b]);
+  if (collide) { seterr(err, cap, "output index function not injective (reading C-5)"); { free(sp); return -2; } }
+  { free(sp); return 0; }
 }
 
 /* Sampled evaluation at n_points cc coordinates (points: n_points × D full
@@ -442,12 +446,13 @@ int mdho_eval(const int64_t* enc, int64_t n, const double* fp, int nfp,
 int mdho_eval_points(const int64_t* enc, int64_t n, const double* fp, int nfp,
                      const void* const* in, int64_t np, const int64_t* points,
                      int64_t* lin, double* vf, int64_t* vi, int nthreads, char* err, int cap) {
-  ospec s;
-  if (prepare(enc, n, fp, nfp, &s, err, cap)) return -1;
+  ospec* sp = (ospec*)calloc(1, sizeof(ospec));   /* ~0.7 MB: heap, not stack */
+  if (!sp) { seterr(err, cap, "oom"); return -1; }
+  if (prepare(enc, n, fp, nfp, sp, err, cap)) { free(sp); return -1; }
   for (int64_t p = 0; p < np; ++p)
-    for (int t = 0; t < s.ncc; ++t) {
-      int64_t v = points[p * s.D + s.cc[t]];
-      if (v < 0 || v >= s.size[s.cc[t]]) { seterr(err, cap, "point out of range"); return -1; }
+    for (int t = 0; t < sp->ncc; ++t) {
+      int64_t v = points[p * sp->D + sp->cc[t]];
+      if (v < 0 || v >= sp->size[sp->cc[t]]) { seterr(err, cap, "point out of range"); { free(sp); return -1; } }
     }
 #ifdef _OPENMP
   if (nthreads > 0) omp_set_num_threads(nthreads);
@@ -457,20 +462,20 @@ int mdho_eval_points(const int64_t* enc, int64_t n, const double* fp, int nfp,
     int64_t idx[O_MAXD];
     otuple y;
     memset(idx, 0, sizeof(idx));
-    for (int t = 0; t < s.ncc; ++t) idx[s.cc[t]] = points[p * s.D + s.cc[t]];
+    for (int t = 0; t < sp->ncc; ++t) idx[sp->cc[t]] = points[p * sp->D + sp->cc[t]];
     memset(&y, 0, sizeof(y));
     int64_t keep[O_MAXD];
     memcpy(keep, idx, sizeof(keep));
-    fold(&s, in, idx, keep, 0, &y);
-    for (int b = 0; b < s.nout; ++b) {
-      const obuf* B = &s.b[s.nin + b];
-      int c = (s.f == S_PRL) ? b : 0;
-      lin[b * np + p] = lin_index(&s, B, 0, idx);
+    fold(sp, in, idx, keep, 0, &y);
+    for (int b = 0; b < sp->nout; ++b) {
+      const obuf* B = &sp->b[sp->nin + b];
+      int c = (sp->f == S_PRL) ? b : 0;
+      lin[b * np + p] = lin_index(sp, B, 0, idx);
       if (is_float_t(B->dtype)) vf[b * np + p] = y.f[c];
       else vi[b * np + p] = y.i[c];
     }
   }
-  return 0;
+  { free(sp); return 0; }
 }
 
 /* Ordered ⊗-fold of two partial results given as tuples (used by the homomorphism
@@ -478,14 +483,14 @@ int mdho_eval_points(const int64_t* enc, int64_t n, const double* fp, int nfp,
  * lf/li, rf/ri: per component (3) fp64 / int64.  Writes the result into lf/li.   */
 int mdho_combine_tuple(int op, int f, int kind, double* lf, int64_t* li, const double* rf,
                        const int64_t* ri) {
-  ospec s;
-  memset(&s, 0, sizeof(s));
-  s.f = f;
-  s.kind = kind;
+  static __thread ospec* sp = NULL;     /* combine() reads only f and kind */
+  if (!sp && !(sp = (ospec*)calloc(1, sizeof(ospec)))) return -1;
+  sp->f = f;
+  sp->kind = kind;
   otuple l, r, res;
   for (int c = 0; c < 3; ++c) { l.f[c] = lf[c]; l.i[c] = li[c]; r.f[c] = rf[c]; r.i[c] = ri[c]; }
   res = l;
-  combine(&s, op, &l, &r, &res);
+  combine(sp, op, &l, &r, &res);
   for (int c = 0; c < 3; ++c) { lf[c] = res.f[c]; li[c] = res.i[c]; }
   return 0;
 }

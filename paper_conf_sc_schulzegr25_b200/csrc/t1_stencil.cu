@@ -8,6 +8,8 @@
 // element comes from HBM about once (A2); f = Σ_a w_a·x_a (reading C-16) in fp32
 // with FMA (reading C-13).  HBM-bound: ≈8.05 B per output point for Jacobi3D.
 #include <algorithm>
+#include <type_traits>
+#include <vector>
 
 #include "kcommon.cuh"
 
@@ -141,6 +143,176 @@ __global__ void __launch_bounds__(128) t1_j3d7_kernel(const __grid_constant__ J7
   }
 }
 
+// ---- dense 2-D box stencil (H×W window, e.g. Gaussian_2D 5×5, Fig 3) -------
+// Each thread owns 4 consecutive x outputs and marches y over a y-chunk with a register
+// window of the last H input rows (4+W-1 values each): a y step loads ONE new row segment
+// (two 16-byte loads for W = 5) and does 4·|accesses| FMAs; rows are re-read only across
+// chunk boundaries (H-1 halo rows per chunk, L2 hits).  Absent window taps (a sparse
+// stencil inside its bounding box) are skipped through the mask, so the arithmetic is
+// exactly Σ_a w_a·x_a over the spec's accesses (reading C-16/C-31), fp32 FMA.
+struct Box2Params {
+  const float* u;
+  float* v;
+  int64_t b0;              // element offset of window tap (0,0) at the origin
+  int64_t Ly;              // input row stride (x stride 1)
+  int64_t ob, oLy;         // output (x stride 1)
+  int X, Y, ychunk;
+  uint64_t mask;           // bit r*W+s: tap (r,s) present
+  float w[49];             // w[r*W+s]
+};
+
+template <int H, int W, bool DENSE>
+__global__ void __launch_bounds__(128) t1_box2d_kernel(const __grid_constant__ Box2Params P) {
+  constexpr int NW = 4 + W - 1;
+  const int x0 = (blockIdx.x * blockDim.x + threadIdx.x) * 4;
+  if (x0 >= P.X) return;
+  const int y0 = blockIdx.y * P.ychunk;
+  const int y1 = min(P.Y, y0 + P.ychunk);
+  const int nv = min(4, P.X - x0);                       // valid outputs of this thread
+  const bool vec = nv == 4 && ((P.b0 + x0) & 3) == 0 && (P.Ly & 3) == 0;
+  const bool ovec = nv == 4 && ((P.ob + x0) & 3) == 0 && (P.oLy & 3) == 0;
+  const float* pin = P.u + P.b0 + x0 + (int64_t)y0 * P.Ly;
+  float* po = P.v + P.ob + x0 + (int64_t)y0 * P.oLy;
+  float w[H * W];
+#pragma unroll
+  for (int k = 0; k < H * W; ++k) w[k] = P.w[k];
+  // window ring: slot (ph + r) % H holds window row r at phase ph; unrolling the y loop by H
+  // makes every slot index a compile-time constant (no register moves)
+  float win[H][NW];
+  auto load_row = [&](const float* p, float* r) {
+    if (vec) {
+#pragma unroll
+      for (int k = 0; k + 4 <= NW; k += 4) {
+        const float4 a = __ldg(reinterpret_cast<const float4*>(p + k));
+        r[k] = a.x; r[k + 1] = a.y; r[k + 2] = a.z; r[k + 3] = a.w;
+      }
+      if (NW % 4 >= 2) {
+        const float2 a = __ldg(reinterpret_cast<const float2*>(p + (NW & ~3)));
+        r[NW & ~3] = a.x; r[(NW & ~3) + 1] = a.y;
+      }
+      if (NW % 2) r[NW - 1] = __ldg(p + NW - 1);
+    } else {
+#pragma unroll
+      for (int k = 0; k < NW; ++k) r[k] = k < nv + W - 1 ? __ldg(p + k) : 0.f;
+    }
+  };
+  // step at phase PH: load window row H-1 into slot (PH + H - 1) % H, compute, store
+  auto step = [&](auto ph) {
+    constexpr int PH = decltype(ph)::value;
+    load_row(pin + (int64_t)(H - 1) * P.Ly, win[(PH + H - 1) % H]);
+    float o[4] = {0.f, 0.f, 0.f, 0.f};
+#pragma unroll
+    for (int r = 0; r < H; ++r)
+#pragma unroll
+      for (int s = 0; s < W; ++s)
+        if (DENSE || ((P.mask >> (r * W + s)) & 1))
+#pragma unroll
+          for (int j = 0; j < 4; ++j) o[j] = fmaf(w[r * W + s], win[(PH + r) % H][j + s], o[j]);
+    if (ovec) {
+      *reinterpret_cast<float4*>(po) = make_float4(o[0], o[1], o[2], o[3]);
+    } else {
+#pragma unroll
+      for (int j = 0; j < 4; ++j)
+        if (j < nv) po[j] = o[j];
+    }
+    pin += P.Ly;
+    po += P.oLy;
+  };
+#pragma unroll
+  for (int r = 0; r < H - 1; ++r) load_row(pin + (int64_t)r * P.Ly, win[r]);
+  int y = y0;
+  for (; y + H <= y1; y += H) {
+    step(std::integral_constant<int, 0>{});
+    step(std::integral_constant<int, 1>{});
+    step(std::integral_constant<int, 2>{});
+    if constexpr (H > 3) {
+      step(std::integral_constant<int, 3>{});
+      step(std::integral_constant<int, 4>{});
+    }
+  }
+  // tail (< H rows): phases 0, 1, … continue the ring from phase 0
+  if (y < y1) step(std::integral_constant<int, 0>{});
+  if (y + 1 < y1) step(std::integral_constant<int, 1>{});
+  if constexpr (H > 3) {
+    if (y + 2 < y1) step(std::integral_constant<int, 2>{});
+    if (y + 3 < y1) step(std::integral_constant<int, 3>{});
+  }
+}
+
+// Recognise a dense 2-D window: one fp32 input buffer, ≤ 49 accesses sharing the linear
+// part with x stride 1, taps inside an H×W box, H = W ∈ {3, 5}; exactly two non-degenerate
+// dims (y, x).  auxi = {-2, dy, dx, H, W, b0, tap index per access ...}.
+static bool detect_box2d(Plan* p) {
+  if (p->n_in != 1 || p->f != MDH_F_STENCIL || p->in[0].dtype != MDH_F32 || p->out[0].dtype != MDH_F32) return false;
+  int dims[2], nd = 0;
+  for (int d = 0; d < p->D; ++d)
+    if (p->size[d] > 1) { if (nd == 2) return false; dims[nd++] = d; }
+  if (nd != 2) return false;
+  const int dy = dims[0], dx = dims[1];
+  const Buf& B = p->in[0];
+  for (int a = 1; a < B.nacc; ++a)
+    for (int d = 0; d < p->D; ++d)
+      if (B.acc[a].L[d] != B.acc[0].L[d]) return false;
+  const int64_t Ly = B.acc[0].L[dy];
+  if (B.acc[0].L[dx] != 1 || Ly < 8 || p->out[0].acc[0].L[dx] != 1) return false;
+  // decompose each tap offset relative to the smallest base into (r, s), 0 <= s < Ly/2
+  int64_t bmin = INT64_MAX;
+  for (int a = 0; a < B.nacc; ++a) bmin = std::min(bmin, B.acc[a].base);
+  int rmin = 1 << 30, rmax = -1, smin = 1 << 30, smax = -(1 << 30);
+  std::vector<std::pair<int64_t, int64_t>> rs;
+  for (int a = 0; a < B.nacc; ++a) {
+    const int64_t d = B.acc[a].base - bmin;
+    int64_t r = (d + Ly / 2) / Ly, s = d - r * Ly;
+    rs.push_back({r, s});
+    rmin = std::min<int>(rmin, (int)r); rmax = std::max<int>(rmax, (int)r);
+    smin = std::min<int>(smin, (int)s); smax = std::max<int>(smax, (int)s);
+  }
+  const int H = rmax - rmin + 1, W = smax - smin + 1;
+  if (!((H == 3 && W == 3) || (H == 5 && W == 5)) || B.nacc < 4) return false;
+  std::vector<int> seen(H * W, 0);
+  p->auxi = {-2, dy, dx, H, W, bmin + rmin * Ly + smin};
+  for (auto& t : rs) {
+    const int k = (int)(t.first - rmin) * W + (int)(t.second - smin);
+    if (seen[k]++) return false;              // duplicate tap: keep the literal generic path
+    p->auxi.push_back(k);
+  }
+  return true;
+}
+
+static mdh_status launch_box2d(const Plan& p, const void* const* in, void* const* out, cudaStream_t st) {
+  Box2Params P;
+  memset(&P, 0, sizeof(P));
+  const int dy = (int)p.auxi[1], dx = (int)p.auxi[2], H = (int)p.auxi[3], W = (int)p.auxi[4];
+  const Buf& B = p.in[0];
+  const Access& O = p.out[0].acc[0];
+  P.u = (const float*)in[0];
+  P.v = (float*)out[0];
+  P.b0 = p.auxi[5];
+  P.Ly = B.acc[0].L[dy];
+  P.ob = O.base;
+  P.oLy = O.L[dy];
+  P.X = (int)p.size[dx];
+  P.Y = (int)p.size[dy];
+  for (int a = 0; a < B.nacc; ++a) {
+    const int k = (int)p.auxi[6 + a];
+    P.mask |= 1ull << k;
+    P.w[k] = (float)p.fparams[a];
+  }
+  // y-chunk: forced tile knob zchunk, else 16 rows (measured 30.8 µs at 4096², 32: 31.7, 64: 47) (the table's T1 entries are Jacobi's z-chunks)
+  int yc = p.tiles.source.find("forced") != std::string::npos && p.tiles.zchunk > 0 ? p.tiles.zchunk : 16;
+  if (yc > P.Y) yc = P.Y;
+  P.ychunk = yc;
+  const int tx = 64;
+  dim3 grid((unsigned)((P.X + 4 * tx - 1) / (4 * tx)), (unsigned)((P.Y + yc - 1) / yc));
+  const bool dense = P.mask == (H * W == 64 ? ~0ull : (1ull << (H * W)) - 1);
+  if (H == 5 && dense) t1_box2d_kernel<5, 5, true><<<grid, tx, 0, st>>>(P);
+  else if (H == 5) t1_box2d_kernel<5, 5, false><<<grid, tx, 0, st>>>(P);
+  else if (dense) t1_box2d_kernel<3, 3, true><<<grid, tx, 0, st>>>(P);
+  else t1_box2d_kernel<3, 3, false><<<grid, tx, 0, st>>>(P);
+  (void)W;
+  return post_launch("t1_box2d_kernel");
+}
+
 // Recognise the 7-point cross: one fp32 input buffer, 7 accesses sharing the linear part
 // (x stride 1), shifts = centre ± one unit in exactly one of x, y, z.  Stores in auxi:
 // [dz_dim, dy_dim, dx_dim, centre access, index of access for xm,xp,ym,yp,zm,zp].
@@ -182,6 +354,11 @@ mdh_status prepare_t1(Plan* p) {
     p->ws_kernel = 0;
     p->t4_variant = 0;
     p->why += " [7-point cross register-queue kernel]";
+    return MDH_OK;
+  }
+  if (detect_box2d(p)) {
+    p->ws_kernel = 0;
+    p->why += " [2-D box-window register kernel]";
     return MDH_OK;
   }
   // fast path: fp32 inputs, <= 3 non-degenerate dims, <= 32 accesses; else generic
@@ -234,6 +411,7 @@ static mdh_status launch_j3d7(const Plan& p, const void* const* in, void* const*
 }
 
 mdh_status launch_t1(const Plan& p, const void* const* in, void* const* out, void*, cudaStream_t st) {
+  if (!p.auxi.empty() && p.auxi[0] == -2) return launch_box2d(p, in, out, st);
   if (!p.auxi.empty()) return launch_j3d7(p, in, out, st);
   T1Params P;
   memset(&P, 0, sizeof(P));
@@ -272,7 +450,7 @@ mdh_status launch_t1(const Plan& p, const void* const* in, void* const* out, voi
   P.out = out[0];
   P.odt = p.out[0].dtype;
   const int bx = 32, by = 8;
-  int zc = p.tiles.zchunk > 0 ? p.tiles.zchunk : 32;
+  int zc = p.tiles.zchunk > 0 ? p.tiles.zchunk : 16;
   if (P.Z < zc) zc = (int)P.Z;
   P.zchunk = zc;
   dim3 block(bx, by);

@@ -17,7 +17,8 @@ import threading
 
 import numpy as np
 
-MAX_D, MAX_RANK, MAX_ACC, MAX_BUFS = 10, 8, 8, 32
+MAX_D, MAX_RANK, MAX_ACC, MAX_BUFS = 10, 8, 32, 32
+ABI_VERSION = 2                    # include/mdh.h MDH_ABI_VERSION
 HERE = os.path.dirname(os.path.abspath(__file__))
 LIB_PATH = os.path.join(HERE, "libmdh.so")
 
@@ -97,6 +98,8 @@ def lib():
                          "mdh_combine_partials", "mdh_destroy", "mdh_comm_unique_id", "mdh_comm_init",
                          "mdh_comm_destroy"):
                 getattr(L, name).restype = ctypes.c_int
+            if L.mdh_abi_version() != ABI_VERSION:
+                raise RuntimeError(f"{LIB_PATH}: ABI version {L.mdh_abi_version()} != {ABI_VERSION} (stale build?)")
             _lib = L
     return _lib
 

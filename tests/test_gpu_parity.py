@@ -110,6 +110,29 @@ def test_jacobi3d_full_size_sampled_and_closed_forms():
     assert np.abs(got[0].astype(np.float64) - g["constant_field_2_0"]).max() <= 1e-4 * 2.0 * 2.0 * 1.67
 
 
+@pytest.mark.parametrize("IJ", [(1, 1), (3, 5), (17, 33), (224, 224), (129, 1030)])
+def test_gaussian2d(IJ):
+    """Gaussian_2D 5×5 (reading C-31; Fig 3) on the 2-D box-window T1 kernel:
+    ragged x (non-multiple of 4, unaligned rows) and y-chunk tails."""
+    I, J = IJ
+    spec = S.gaussian2d(I, J)
+    x = G.gaussian2d_inputs(I, J)
+    got, p = run_gpu(spec, x)
+    assert p.template == "T1_stencil"
+    assert "box-window" in p.describe()["why"] or I * J < 4
+    assert_close_full(spec, x, got, 1e-4, kind="rel")
+
+
+def test_gaussian2d_full_size_closed_forms():
+    I = J = 4096
+    spec = S.gaussian2d(I, J)
+    got, _ = run_gpu(spec, G.gaussian2d_inputs(I, J, "constant"))
+    assert np.allclose(got[0], 3.0, rtol=1e-6, atol=0)
+    x = G.gaussian2d_inputs(I, J)
+    got, _ = run_gpu(spec, x)
+    assert_close_points(spec, x, got, 1e-4, n=20000, kind="rel")
+
+
 @pytest.mark.parametrize("K", [1, 3, 1000])
 def test_jacobi1d(K):
     spec = S.jacobi1d(K)

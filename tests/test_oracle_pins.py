@@ -153,6 +153,26 @@ def test_jacobi3d_vs_numpy_slicing():
     assert np.allclose(v, ref, rtol=0, atol=1e-13)
 
 
+def test_gaussian2d_closed_forms_and_scipy():
+    """Gaussian_2D (reading C-31): dyadic weights k/256 make the closed forms exact in fp64 —
+    a constant field is reproduced, the symmetric window maps a linear field x + 2y to its
+    value at the window centre; random images agree with scipy's 'valid' correlation."""
+    import scipy.signal
+    I, J = 9, 13
+    sp = S.gaussian2d(I, J)
+    assert abs(sum(sp["fparams"]) - 1.0) == 0.0
+    v = oracle.evaluate(sp, G.gaussian2d_inputs(I, J, "constant"))[0]
+    assert v.shape == (I, J) and np.all(v == 3.0)
+    v = oracle.evaluate(sp, G.gaussian2d_inputs(I, J, "linear"))[0]
+    jj, ii = np.meshgrid(np.arange(J), np.arange(I))
+    assert np.array_equal(v, (jj + 2) + 2.0 * (ii + 2))
+    img = G.gaussian2d_inputs(I, J)[0]
+    w = np.outer(S.GAUSS5, S.GAUSS5) / 256.0
+    ref = scipy.signal.correlate2d(img.astype(np.float64), w, mode="valid")
+    v = oracle.evaluate(sp, [img])[0]
+    assert np.allclose(v, ref, rtol=0, atol=1e-14)
+
+
 def test_jacobi1d_three_accesses():
     K = 1000
     vin = G.rng(9).uniform(0, 1, K + 2).astype(np.float32)
