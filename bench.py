@@ -100,6 +100,11 @@ def workload(name, world=1, rank=0):
         spec = S.matvec(4096, 4096)
         return dict(spec=spec, inputs=lambda: G.gen_inputs(spec, 2100), work=4.0 * (4096 * 4096 + 4096 + 4096),
                     unit="GB/s", scale=1e9, bound="hbm", dtype="f32", desc="MatVec 4096^2 fp32 (Fig 3 P:514)")
+    if name == "mcc_caps_bf16":
+        spec = S.mcc_caps(16, 112, 112, 64, 7, 7, 3, dtype="bf16")
+        return dict(spec=spec, inputs=lambda: G.gen_inputs(spec, 4300), work=2.0 * 16 * 112 * 112 * 64 * 16 * 588,
+                    unit="TFLOP/s", scale=1e12, bound="tensor", dtype="bf16",
+                    desc="MCC_Caps 16x230x230x3x4x4 * 64x7x7x3x4x4 bf16 (Fig 3 P:530; reading C-33)")
     if name == "prefix_sum_f32":
         spec = S.prefix_sum([1 << 26], 0)
         return dict(spec=spec, inputs=lambda: G.gen_inputs(spec, 6100, "positive"), work=8.0 * (1 << 26),
@@ -119,7 +124,7 @@ def workload(name, world=1, rank=0):
 
 
 SUITE = ["dot_f32", "dot_i32", "dot_f32_2^28", "matvec_f32", "matvec_4096", "jacobi3d", "gaussian2d", "matmul_f32",
-         "matmul_bf16", "ccsd_bf16", "mcc_bf16", "prl_A", "prl_B", "prefix_sum_f32", "mbbs_f32"]
+         "matmul_bf16", "ccsd_bf16", "mcc_bf16", "mcc_caps_bf16", "prl_A", "prl_B", "prefix_sum_f32", "mbbs_f32"]
 
 
 def roofline(w, seconds, pk):

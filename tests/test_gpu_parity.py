@@ -492,3 +492,34 @@ def test_t4_scatter_epilogues(case):
         assert_close_points(spec, x, got, 1e-2, n=50000, kind="scale")
     else:
         assert_close_full(spec, x, got, 1e-2, kind="scale")
+
+
+# ------------------------------------------- F4: the remaining Fig 3 workloads (paper sizes)
+PAPER_CASES = {
+    # name: (spec builder, input seed, sampled points or None = full check)
+    "matmul_1024": (lambda: S.matmul(1024, 1024, 1024, "f32"), 7001, 20000),
+    "matmul_1x2048x1000": (lambda: S.matmul(1, 1000, 2048, "f32"), 7002, None),
+    "matmul_t_10x500x64": (lambda: S.matmul_t(10, 500, 64, "f32"), 7003, None),
+    "bmatmul_16x10x500x64": (lambda: S.bmatmul(16, 10, 500, 64, "f32"), 7004, None),
+    "ccsd_inp1_sd2": (lambda: S.ccsd_sd2(), 7005, 20000),
+    "ccsd_inp2_sd1x": (lambda: S.ccsd_sd1x(24, 16, 24, 16, 16, 24, 16), 7006, 20000),
+    "mcc_caps_small": (lambda: S.mcc_caps(2, 5, 3, 4, 3, 3, 3), 7007, None),
+    "mcc_caps_inp2": (lambda: S.mcc_caps(1, 112, 112, 64, 7, 7, 3), 7008, 5000),
+    "mcc_caps_small_bf16": (lambda: S.mcc_caps(2, 5, 3, 4, 3, 3, 3, dtype="bf16"), 7009, None),
+    "mcc_caps_inp2_bf16": (lambda: S.mcc_caps(1, 112, 112, 64, 7, 7, 3, dtype="bf16"), 7010, 5000),
+}
+
+
+@pytest.mark.parametrize("case", sorted(PAPER_CASES))
+def test_fig3_paper_sizes(case):
+    """MatMul (1024³; 1×2048 · 2048×1000), MatMul^T, bMatMul, CCSD(T) Inp.1/Inp.2 and MCC_Caps
+    (Fig 3; readings C-22, C-33) through whatever template the planner picks."""
+    build, seed, n = PAPER_CASES[case]
+    spec = build()
+    x = G.gen_inputs(spec, seed)
+    got, p = run_gpu(spec, x)
+    tol = 1e-2 if spec["inputs"][0]["dtype"] == "bf16" else 1e-4
+    if n is None:
+        assert_close_full(spec, x, got, tol, kind="scale")
+    else:
+        assert_close_points(spec, x, got, tol, n=n, kind="scale")

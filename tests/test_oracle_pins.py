@@ -220,6 +220,30 @@ def test_mcc_vs_torch_conv2d():
     assert np.allclose(res, ref, rtol=0, atol=1e-13)
 
 
+def test_mcc_caps_vs_strided_einsum():
+    """MCC_Caps (reading C-33): numpy strided-window view of the image + einsum over
+    (r, s, c, l) with the 4×4 capsule matrix product; with 1×1 capsules it is MCC and
+    matches torch conv2d."""
+    N, P, Q, K, R, Sx, C = 2, 3, 2, 3, 3, 3, 2
+    sp = S.mcc_caps(N, P, Q, K, R, Sx, C, 2, 3, 4)
+    img, flt = G.gen_inputs(sp, 4200)
+    res = oracle.evaluate(sp, [img, flt])[0]
+    X = img.astype(np.float64)
+    win = np.lib.stride_tricks.sliding_window_view(X, (R, Sx), axis=(1, 2))[:, ::2, ::2]
+    win = win[:, :P, :Q]                                   # [n,p,q,c,i,l,r,s]
+    ref = np.einsum("npqcilrs,krsclj->npqkij", win, flt.astype(np.float64))
+    assert res.shape == ref.shape
+    assert np.allclose(res, ref, rtol=0, atol=1e-13)
+    torch = pytest.importorskip("torch")
+    sp1 = S.mcc_caps(N, P, Q, K, R, Sx, C, 1, 1, 1)
+    img1, flt1 = G.gen_inputs(sp1, 4210)
+    r1 = oracle.evaluate(sp1, [img1, flt1])[0][..., 0, 0]
+    x = torch.from_numpy(img1[..., 0, 0].astype(np.float64)).permute(0, 3, 1, 2)
+    w = torch.from_numpy(flt1[..., 0, 0].astype(np.float64)).permute(0, 3, 1, 2)
+    ref1 = torch.nn.functional.conv2d(x, w, stride=2)[:, :, :P, :Q].permute(0, 2, 3, 1).numpy()
+    assert np.allclose(r1, ref1, rtol=0, atol=1e-13)
+
+
 # --------------------------------------------------------------- PRL (C5)
 def _prl_numpy(new, db, dbid, wa, wd, op):
     """Independent vectorised formulation (SURVEY §8(c).4 PRL row): broadcast compare,
