@@ -71,6 +71,7 @@ struct Tiles {
   int implicit = 0;                   // T4 A operand when not 2-D: 0 auto, 1 N-d TMA box (implicit
                                       // GEMM), 2 in-kernel cp.async gather, 3 gather pre-pass
   int epi = 0;                        // T4 scatter epilogue: 0 auto, 1 never the bulk-run (EPI 3) kernel
+  int krot = 0;                       // T4 k-block rotation per tile (1 = on)
   std::string source = "default";
 };
 

@@ -83,6 +83,15 @@ struct Params {
   int nstg;                         // staging buffers per epilogue warp (1 or 2)
   int e3flip;                       // EPI 3 bank-conflict-free staging order (tile knob epi=2: off)
   int bres;                         // EPI 3: B of the current N-tile resident in shared memory
+  // A via TMA im2col (convolution operands, MCC Listing 12): A[(n,p,q), (r,s,c)] =
+  // img[n, σh·p + r, σw·q + s, c]; the tensor map walks 128 output pixels (q, then p, then
+  // n) with traversal strides (σw, σh) and applies the filter tap (s, r) as im2col offsets
+  int a_im2col;
+  int ic_C, ic_P, ic_Q, ic_S, ic_sh, ic_sw;
+  // k-block rotation: tile t walks its k-range starting at a t-dependent offset, so the
+  // CTAs of a wave do not all request the same B rows (MCC: 49 M-tiles share each filter
+  // tile) from the same L2 lines at the same time; the fp32 sum order changes only
+  int krot;
 };
 
 constexpr int AG_WARPS = 4, AG_THREADS = AG_WARPS * 32, KOFF_MAX = 2048;
@@ -98,6 +107,12 @@ __device__ __forceinline__ void cp_async_commit() { asm volatile("cp.async.commi
 template <int N>
 __device__ __forceinline__ void cp_async_wait() { asm volatile("cp.async.wait_group %0;" ::"n"(N) : "memory"); }
 __device__ __forceinline__ void fence_proxy_async() { asm volatile("fence.proxy.async.shared::cta;" ::: "memory"); }
+
+__device__ __forceinline__ int krotate(const Params& P, int kb, int kb0, int kb1, int salt) {
+  if (!P.krot) return kb;
+  const int n = kb1 - kb0;
+  return kb0 + (kb - kb0 + (salt * 5) % n) % n;
+}
 
 __device__ __forceinline__ void unit_decode(const Params& P, int u, int* t, int* kb0, int* kb1, int* slot) {
   if (u < P.nfull) {
@@ -163,6 +178,27 @@ __device__ __forceinline__ void tma_load_2d(uint32_t dst, const CUtensorMap* map
   asm volatile(
       "cp.async.bulk.tensor.2d.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1, {%3, %4}], [%2];" ::"r"(dst),
       "l"((uint64_t)map), "r"(bar), "r"(c0), "r"(c1)
+      : "memory");
+}
+// im2col A tile: coordinates of the first output pixel's window origin and the tap offsets
+__device__ __forceinline__ void im2col_coords(const Params& P, int64_t m0, int k0, int* c, uint16_t* off) {
+  const int64_t pq = (int64_t)P.ic_P * P.ic_Q;
+  const int n = (int)(m0 / pq), rem = (int)(m0 % pq);
+  const int p = rem / P.ic_Q, q = rem % P.ic_Q;
+  const int sc = P.ic_S * P.ic_C;
+  const int r = k0 / sc, s = (k0 / P.ic_C) % P.ic_S;
+  c[0] = k0 % P.ic_C;
+  c[1] = P.ic_sw * q;
+  c[2] = P.ic_sh * p;
+  c[3] = n;
+  off[0] = (uint16_t)s;
+  off[1] = (uint16_t)r;
+}
+__device__ __forceinline__ void tma_load_im2col(uint32_t dst, const CUtensorMap* map, uint32_t bar, const int* c,
+                                                const uint16_t* off) {
+  asm volatile(
+      "cp.async.bulk.tensor.4d.shared::cluster.global.im2col.mbarrier::complete_tx::bytes [%0], [%1, {%3, %4, %5, %6}], [%2], {%7, %8};" ::"r"(dst),
+      "l"((uint64_t)map), "r"(bar), "r"(c[0]), "r"(c[1]), "r"(c[2]), "r"(c[3]), "h"(off[0]), "h"(off[1])
       : "memory");
 }
 __device__ __forceinline__ void tma_load_nd(uint32_t dst, const CUtensorMap* map, uint32_t bar, int rank, const int* c) {
@@ -344,9 +380,14 @@ __global__ void __launch_bounds__(AG ? THREADS + AG_THREADS : THREADS, 1)
           const uint32_t fb = full0 + 8 * stage;
           mbar_expect_tx(fb, AG ? b_stage : (bres ? A_BYTES : A_BYTES + b_stage));
           const uint32_t a_dst = smem_u32(sA + stage * A_BYTES), b_dst = smem_u32(sB + stage * b_stage);
-          const int k0 = kb * BK;
+          const int k0 = krotate(P, kb, kb0, kb1, mb) * BK;
           if (AG) {
             // A arrives from the gather warps
+          } else if (P.a_im2col) {
+            int cr[4];
+            uint16_t off[2];
+            im2col_coords(P, m0, k0, cr, off);
+            tma_load_im2col(a_dst, &mapA, fb, cr, off);
           } else if (P.a_box) {               // implicit GEMM: one N-d box {64 k*, …1…, 128 g*}
             int cr[5];
             box_coords(P.abox, m0, k0, cr);
@@ -443,7 +484,7 @@ __global__ void __launch_bounds__(AG ? THREADS + AG_THREADS : THREADS, 1)
       for (int kb = kb0; kb < kb1; ++kb, ++g) {
         mbar_wait(empty0 + 8 * stage, phase ^ 1);
         const uint32_t base = smem_u32(sA + stage * A_BYTES);
-        const int kc = kb * (BK / 8) + ch;
+        const int kc = krotate(P, kb, kb0, kb1, (int)mb) * (BK / 8) + ch;
         const int64_t ko = kc < P.nkc ? s_koff[kc] : -1;
 #pragma unroll
         for (int i = 0; i < 8; ++i) {
@@ -755,6 +796,13 @@ __device__ __forceinline__ void tma_load_2d_cg2(uint32_t dst, const CUtensorMap*
       "l"((uint64_t)map), "r"(bar_cluster), "r"(c0), "r"(c1)
       : "memory");
 }
+__device__ __forceinline__ void tma_load_im2col_cg2(uint32_t dst, const CUtensorMap* map, uint32_t bar_cluster, const int* c,
+                                                    const uint16_t* off) {
+  asm volatile(
+      "cp.async.bulk.tensor.4d.im2col.cta_group::2.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1, {%3, %4, %5, %6}], [%2], {%7, %8};" ::"r"(dst),
+      "l"((uint64_t)map), "r"(bar_cluster), "r"(c[0]), "r"(c[1]), "r"(c[2]), "r"(c[3]), "h"(off[0]), "h"(off[1])
+      : "memory");
+}
 __device__ __forceinline__ void mma_bf16_cg2(uint32_t d_tmem, uint64_t a, uint64_t b, uint32_t idesc, uint32_t acc) {
   asm volatile(
       "{\n\t.reg .pred p;\n\tsetp.ne.b32 p, %4, 0;\n\t"
@@ -827,8 +875,13 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(THREADS, 1)
           if (leader) mbar_expect_tx(full0 + 8 * stage, 2 * STAGE2_BYTES);
           else mbar_arrive_cluster(fb_leader);
           const uint32_t a_dst = smem_u32(sA + stage * A2_BYTES), b_dst = smem_u32(sB + stage * B2_BYTES);
-          const int k0 = kb * BK;
-          if (P.a_mn_major) {
+          const int k0 = krotate(P, kb, kb0, kb1, t / P.tiles_n) * BK;
+          if (P.a_im2col) {
+            int cr[4];
+            uint16_t off[2];
+            im2col_coords(P, m0, k0, cr, off);
+            tma_load_im2col_cg2(a_dst, &mapA, fb_leader, cr, off);
+          } else if (P.a_mn_major) {
             tma_load_2d_cg2(a_dst, &mapA, fb_leader, m0, k0);
             tma_load_2d_cg2(a_dst + 8192, &mapA, fb_leader, m0 + 64, k0);
           } else {
@@ -1176,6 +1229,10 @@ struct T4State {
   t4::Params P;
   int cg = 1;      // 1: one SM per 128×256 tile; 2: SM pair per 256×256 tile
   bool ag = false; // A staged by the kernel's gather warps (no A tensor map, no pre-pass)
+  bool ic = false;  // A through a TMA im2col map
+  uint64_t ic_dims[4];
+  int ic_upper[2];
+  uint32_t ic_estr[4];
   int epi = 1;      // 0 row-major C, 1 per-element scatter, 2 run-8 vector scatter, 3 bulk runs
   size_t smem3 = 0; // dynamic shared memory of the EPI 3 kernel
   int tail_parts = 0;   // 1-SM split-K tail: partial tiles in the workspace at tail_off
@@ -1251,6 +1308,54 @@ static bool plan_box(Plan* p, T4State* s) {
   return true;
 }
 
+// TMA im2col planning for A (MCC's img[n, σh·p + r, σw·q + s, c], Listing 12): rank-4 NHWC
+// bf16 buffer, M group (n,) p, q and K group r, s, c in that order, C % 64 == 0.
+static bool plan_im2col(const Plan* p, T4State* s) {
+  const Contraction& c = p->con;
+  const Buf& Ab = p->in[c.a_buf];
+  if (Ab.rank != 4 || Ab.dtype != MDH_BF16 || c.nk != 3 || (c.nm != 2 && c.nm != 3)) return false;
+  const mdh_index_fn& fn = Ab.fn[0];
+  const int dn = c.nm == 3 ? c.md[0] : -1, dp = c.md[c.nm - 2], dq = c.md[c.nm - 1];
+  const int dr = c.kd[0], ds = c.kd[1], dc = c.kd[2];
+  int64_t want[4][MDH_MAX_D] = {};
+  if (dn >= 0) want[0][dn] = 1;
+  want[1][dp] = fn.coeff[1][dp];
+  want[1][dr] = 1;
+  want[2][dq] = fn.coeff[2][dq];
+  want[2][ds] = 1;
+  want[3][dc] = 1;
+  for (int r = 0; r < 4; ++r) {
+    if (fn.offset[r] != 0) return false;
+    for (int d = 0; d < p->D; ++d)
+      if (p->size[d] > 1 && fn.coeff[r][d] != want[r][d]) return false;
+  }
+  const int64_t sh = fn.coeff[1][dp], sw = fn.coeff[2][dq];
+  const int64_t C = Ab.shape[3], H = Ab.shape[1], W = Ab.shape[2];
+  if (sh < 1 || sh > 8 || sw < 1 || sw > 8 || p->size[dc] != C || C % 64) return false;
+  const int64_t P = p->size[dp], Q = p->size[dq], S = p->size[ds];
+  const int64_t uh = sh * (P - 1) - (H - 1), uw = sw * (Q - 1) - (W - 1);
+  if (uh < -128 || uh > 127 || uw < -128 || uw > 127) return false;
+  s->ic_dims[0] = (uint64_t)C;
+  s->ic_dims[1] = (uint64_t)W;
+  s->ic_dims[2] = (uint64_t)H;
+  s->ic_dims[3] = (uint64_t)Ab.shape[0];
+  s->ic_upper[0] = (int)uw;
+  s->ic_upper[1] = (int)uh;
+  s->ic_estr[0] = 1;
+  s->ic_estr[1] = (uint32_t)sw;
+  s->ic_estr[2] = (uint32_t)sh;
+  s->ic_estr[3] = 1;
+  t4::Params& Pp = s->P;
+  Pp.a_im2col = 1;
+  Pp.ic_C = (int)C;
+  Pp.ic_P = (int)P;
+  Pp.ic_Q = (int)Q;
+  Pp.ic_S = (int)S;
+  Pp.ic_sh = (int)sh;
+  Pp.ic_sw = (int)sw;
+  return true;
+}
+
 mdh_status prepare_t4(Plan* p) {
   std::string why;
   if (!t4_supported(*p, &why)) { set_error("T4: %s", why.c_str()); return MDH_ERR_UNSUPPORTED; }
@@ -1264,10 +1369,17 @@ mdh_status prepare_t4(Plan* p) {
   const bool a_2d = a_direct.ok && p->in[c.a_buf].acc[0].base % 8 == 0;
   const bool a_box = !a_2d && p->tiles.implicit == 1 && plan_box(p, s);
   const t4::BoxGen box = s->P.abox;
+  // TMA im2col (implicit 0 = auto or 4): the convolution operand straight from the image
+  t4::Params icp;
+  memset(&icp, 0, sizeof(icp));
+  s->P = icp;
+  const bool a_ic = !a_2d && !a_box && (p->tiles.implicit == 0 || p->tiles.implicit == 4) && plan_im2col(p, s);
+  icp = s->P;
+  s->ic = a_ic;
   // in-kernel gather (implicit 0 = auto or 2): A's K offsets in aligned runs of 8, so each
   // 16-byte chunk of a swizzled A row is one cp.async
   bool a_gather = false;
-  if (!a_2d && !a_box && (p->tiles.implicit == 0 || p->tiles.implicit == 2) && c.K % 8 == 0 &&
+  if (!a_2d && !a_box && !a_ic && (p->tiles.implicit == 0 || p->tiles.implicit == 2) && c.K % 8 == 0 &&
       c.K / 8 <= t4::KOFF_MAX) {
     std::vector<int64_t> tk = t4::table(*p, c.kd, c.nk, p->in[c.a_buf].acc[0]);
     std::vector<int64_t> tm = t4::table(*p, c.md, c.nm, p->in[c.a_buf].acc[0]);
@@ -1281,7 +1393,7 @@ mdh_status prepare_t4(Plan* p) {
     for (size_t i = 0; i < tm.size() && a_gather; ++i)
       if (tm[i] % 8) a_gather = false;
   }
-  if (a_box || a_gather) {
+  if (a_box || a_gather || a_ic) {
     s->a = t4::Layout2D();
     s->a.ok = true;
   } else {
@@ -1295,6 +1407,16 @@ mdh_status prepare_t4(Plan* p) {
   memset(&P, 0, sizeof(P));
   P.a_box = a_box;
   P.abox = box;
+  // (off by default: on MCC conv5_1 it measured 89 vs 98 µs on one box and 103 vs 88.5 on
+  // another; MatMul 4096³ 1048 vs 1266 TFLOP/s)
+  P.krot = p->tiles.krot > 0 ? 1 : 0;
+  P.a_im2col = icp.a_im2col;
+  P.ic_C = icp.ic_C;
+  P.ic_P = icp.ic_P;
+  P.ic_Q = icp.ic_Q;
+  P.ic_S = icp.ic_S;
+  P.ic_sh = icp.ic_sh;
+  P.ic_sw = icp.ic_sw;
   P.M = c.M;
   P.N = c.N;
   P.K = c.K;
@@ -1384,7 +1506,7 @@ mdh_status prepare_t4(Plan* p) {
   P.bn = t4::BN;
   P.nstg = 0;
   P.e3flip = p->tiles.epi != 2;
-  if (s->epi != 0 && !P.out_bf16 && s->cg == 1 && !a_gather && !a_box && !s->b.mn_major && s->tail_parts == 0 &&
+  if (s->epi != 0 && !P.out_bf16 && s->cg == 1 && !a_gather && !a_box && !a_ic && !s->b.mn_major && s->tail_parts == 0 &&
       p->tiles.epi != 1) {
     int64_t L = 1;
     while (L < c.N && cn[(size_t)L] == cn[0] + L) ++L;
@@ -1415,9 +1537,10 @@ mdh_status prepare_t4(Plan* p) {
       }
     }
   }
+  if (s->epi == 3) P.krot = 0;      // the resident-B slots are indexed by the k-block itself
   p->tmaps = s;
   p->t4_variant = 1 + (s->a.permuted ? 2 : 0) + (s->b.permuted ? 4 : 0) + (s->cg == 2 ? 8 : 0) + (a_box ? 16 : 0) +
-                  (a_gather ? 32 : 0) + (s->epi == 2 ? 64 : 0) + (s->epi == 3 ? 128 : 0);
+                  (a_gather ? 32 : 0) + (s->epi == 2 ? 64 : 0) + (s->epi == 3 ? 128 : 0) + (a_ic ? 256 : 0);
   p->ws_kernel = ws;
   p->tiles.bm = s->cg == 2 ? 256 : t4::BM;
   p->tiles.bn = s->epi == 3 ? P.bn : t4::BN;
@@ -1445,6 +1568,38 @@ static PFN_cuTensorMapEncodeTiled_v12000 encode_fn() {
       fn = (PFN_cuTensorMapEncodeTiled_v12000)f;
   });
   return fn;
+}
+
+typedef CUresult (*EncodeIm2colFn)(CUtensorMap*, CUtensorMapDataType, cuuint32_t, void*, const cuuint64_t*,
+                                   const cuuint64_t*, const int*, const int*, cuuint32_t, cuuint32_t, const cuuint32_t*,
+                                   CUtensorMapInterleave, CUtensorMapSwizzle, CUtensorMapL2promotion,
+                                   CUtensorMapFloatOOBfill);
+static EncodeIm2colFn encode_im2col_fn() {
+  static EncodeIm2colFn fn = nullptr;
+  static std::once_flag once;
+  std::call_once(once, [] {
+    void* f = nullptr;
+    cudaDriverEntryPointQueryResult q;
+    if (cudaGetDriverEntryPoint("cuTensorMapEncodeIm2col", &f, cudaEnableDefault, &q) == cudaSuccess &&
+        q == cudaDriverEntryPointSuccess)
+      fn = (EncodeIm2colFn)f;
+  });
+  return fn;
+}
+
+// im2col map of an NHWC bf16 image: 64 channels × 128 output pixels per load (SWIZZLE_128B
+// rows, the K-major A tile layout); lower corner 0, upper corner so that the traversal
+// visits exactly P (Q) window origins with strides (σh, σw)
+static mdh_status make_im2col_map(CUtensorMap* map, const void* base, const T4State& s) {
+  auto fn = encode_im2col_fn();
+  if (!fn) { set_error("cuTensorMapEncodeIm2col unavailable"); return MDH_ERR_CUDA; }
+  cuuint64_t strides[3] = {s.ic_dims[0] * 2, s.ic_dims[0] * s.ic_dims[1] * 2, s.ic_dims[0] * s.ic_dims[1] * s.ic_dims[2] * 2};
+  int lower[2] = {0, 0};
+  CUresult r = fn(map, CU_TENSOR_MAP_DATA_TYPE_BFLOAT16, 4, const_cast<void*>(base), s.ic_dims, strides, lower, s.ic_upper,
+                  64, 128, s.ic_estr, CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_128B,
+                  CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+  if (r != CUDA_SUCCESS) { set_error("cuTensorMapEncodeIm2col failed (%d)", (int)r); return MDH_ERR_CUDA; }
+  return MDH_OK;
 }
 
 // 2-D bf16 tensor map: inner dim `inner` (unit stride), outer dim `outer` with stride ld
@@ -1527,6 +1682,9 @@ mdh_status launch_t4(const Plan& p, const void* const* in, void* const* out, voi
                     strides, box, estr, CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_128B,
                     CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
     if (r != CUDA_SUCCESS) { set_error("cuTensorMapEncodeTiled (implicit GEMM) failed (%d)", (int)r); return MDH_ERR_CUDA; }
+  } else if (s->ic) {
+    if ((uintptr_t)A % 16) { set_error("T4 im2col: A buffer not 16-byte aligned"); return MDH_ERR_INVALID_ARG; }
+    MDH_TRY(make_im2col_map(&ma, A, *s));
   } else if (s->ag) {
     if ((uintptr_t)A % 16) { set_error("T4 gather: A buffer not 16-byte aligned"); return MDH_ERR_INVALID_ARG; }
     P.Ag = A;

@@ -145,6 +145,7 @@ void apply(Tiles* t, const std::string& k, double v) {
   else if (k == "cluster") t->cluster = iv;
   else if (k == "implicit") t->implicit = iv;
   else if (k == "epi") t->epi = iv;
+  else if (k == "krot") t->krot = iv;
 }
 
 std::string read_file(const char* path) {

@@ -523,3 +523,22 @@ def test_fig3_paper_sizes(case):
         assert_close_full(spec, x, got, tol, kind="scale")
     else:
         assert_close_points(spec, x, got, tol, n=n, kind="scale")
+
+
+@pytest.mark.parametrize("cfg,tile", [((256, 7, 7, 512, 3, 3, 512), None),           # conv5_1, 2-SM
+                                      ((3, 3, 5, 128, 3, 3, 64), None),              # P != Q, ragged M
+                                      ((2, 9, 4, 256, 3, 3, 128), "cluster=1"),      # 1-SM kernel
+                                      ((64, 7, 7, 512, 3, 3, 512), "split=3"),       # 2-SM split-K tail
+                                      ((5, 6, 6, 64, 2, 2, 64), None)])              # 2x2 window
+def test_mcc_im2col_tma(cfg, tile):
+    """T4 A operand through a TMA im2col map (window origin walk with traversal strides,
+    filter taps as im2col offsets; no gather pre-pass, no gather warps)."""
+    spec = S.mcc(*cfg, dtype="bf16")
+    x = G.mcc_inputs(spec)
+    got, p = run_gpu(spec, x, force_tile=tile)
+    v = p.describe()["t4_variant"]
+    assert v & 256, v
+    if np.prod(cfg) > 1e9:
+        assert_close_points(spec, x, got, 1e-2, n=20000, kind="scale")
+    else:
+        assert_close_full(spec, x, got, 1e-2, kind="scale")
