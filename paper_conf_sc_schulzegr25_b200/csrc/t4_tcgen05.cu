@@ -21,6 +21,8 @@
 #include <cudaTypedefs.h>
 
 #include <algorithm>
+#include <cstdio>
+#include <cstdlib>
 #include <vector>
 
 #include "kcommon.cuh"
@@ -92,6 +94,18 @@ struct Params {
   // CTAs of a wave do not all request the same B rows (MCC: 49 M-tiles share each filter
   // tile) from the same L2 lines at the same time; the fp32 sum order changes only
   int krot;
+  // 2-SM stream-K hybrid: tiles [0, nfull) data-parallel (round-robin over the pairs), then
+  // the (tile, k-block) space of the remaining tiles, sk_w = (num_tiles - nfull)·num_kb
+  // k-blocks, cut into sk_pairs equal contiguous ranges, one per pair (0 = off)
+  int sk_pairs;
+  int64_t sk_w;
+  float* skpart;                    // one fp32 256×256 partial tile per pair (coalesced layout)
+  unsigned* skflag;                 // 16 flags per pair (2 CTAs × 8 epilogue warps); zero at rest
+  // diagnostics: per-unit timeline (MDH_T4_TRACE=1; 2-SM kernel), 4 u64 per unit:
+  // {smid << 32 | cluster, first MMA issue, last commit, epilogue done} in ns (%globaltimer)
+  unsigned long long* trace;
+  int trace_n;                      // units the trace buffer holds
+  int c_vec4;                       // row-major C with ldc, cbase ≡ 0 mod 4 and a 16-byte base
 };
 
 constexpr int AG_WARPS = 4, AG_THREADS = AG_WARPS * 32, KOFF_MAX = 2048;
@@ -107,6 +121,17 @@ __device__ __forceinline__ void cp_async_commit() { asm volatile("cp.async.commi
 template <int N>
 __device__ __forceinline__ void cp_async_wait() { asm volatile("cp.async.wait_group %0;" ::"n"(N) : "memory"); }
 __device__ __forceinline__ void fence_proxy_async() { asm volatile("fence.proxy.async.shared::cta;" ::: "memory"); }
+
+__device__ __forceinline__ unsigned long long gtimer() {
+  unsigned long long t;
+  asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+  return t;
+}
+__device__ __forceinline__ unsigned smid() {
+  unsigned r;
+  asm volatile("mov.u32 %0, %%smid;" : "=r"(r));
+  return r;
+}
 
 __device__ __forceinline__ int krotate(const Params& P, int kb, int kb0, int kb1, int salt) {
   if (!P.krot) return kb;
@@ -771,15 +796,62 @@ __global__ void __launch_bounds__(AG ? THREADS + AG_THREADS : THREADS, 1)
 // both CTAs' TMA bytes (cta_group::2 TMA signals the leader); MMA commits are multicast to
 // both CTAs' empty / tmem-full barriers; both epilogues release the accumulator at the
 // leader's tmem-empty barrier.
+// Work schedule of a CTA pair: data-parallel whole tiles u = pair, pair + npairs, … < nfull,
+// then the pair's stream-K range [s_p, s_{p+1}), s_p = p·sk_w / sk_pairs, cut at tile
+// boundaries into segments (tile, kb0, kb1).  Role of a segment: 0 whole tile; 1 producer
+// (kb0 > 0: the partial sum goes to the pair's workspace slot — it is always the pair's
+// FIRST stream-K segment); 2 finisher (kb0 = 0, kb1 < num_kb: the pair's LAST segment; it
+// adds the producers' partials p+1, p+2, … in k order before the store).  Producers run
+// first and finishers last, so a finisher finds its partials (nearly always) published;
+// all pairs are co-resident (persistent grid), so the flag waits cannot deadlock.
+struct SkWork { int t, kb0, kb1, role; };
+struct SkIter {
+  int u, step, nfull, kb;
+  int64_t k, e;
+  __device__ __forceinline__ SkIter(const Params& P, int pair, int npairs) {
+    u = pair;
+    step = npairs;
+    nfull = P.nfull;
+    kb = P.num_kb;
+    k = e = 0;
+    if (P.sk_pairs > 0 && pair < P.sk_pairs) {
+      k = (int64_t)pair * P.sk_w / P.sk_pairs;
+      e = (int64_t)(pair + 1) * P.sk_w / P.sk_pairs;
+    }
+  }
+  __device__ __forceinline__ bool next(SkWork* w) {
+    if (u < nfull) {
+      w->t = u; w->kb0 = 0; w->kb1 = kb; w->role = 0;
+      u += step;
+      return true;
+    }
+    if (k >= e) return false;
+    const int64_t x = k / kb;
+    w->t = nfull + (int)x;
+    w->kb0 = (int)(k - x * kb);
+    const int64_t rem = e - k;
+    w->kb1 = rem < (int64_t)(kb - w->kb0) ? w->kb0 + (int)rem : kb;
+    w->role = (w->kb0 == 0 && w->kb1 == kb) ? 0 : (w->kb0 == 0 ? 2 : 1);
+    k += w->kb1 - w->kb0;
+    return true;
+  }
+};
+
 constexpr int S2 = 6;                          // stages (32 KB each)
 constexpr int A2_BYTES = 128 * BK * 2;         // this CTA's half of A (16 KB)
 constexpr int B2_BYTES = 128 * BK * 2;         // this CTA's half of B (16 KB)
 constexpr int STAGE2_BYTES = A2_BYTES + B2_BYTES;
-constexpr int SMEM2_BYTES = S2 * STAGE2_BYTES + 1024 + 256;
+constexpr int STG2_BYTES = 8 * 32 * 32 * 4;    // epilogue staging: 32×32 fp32 per epilogue warp
+constexpr int SMEM2_BYTES = S2 * STAGE2_BYTES + 1024 + 256 + STG2_BYTES;
 
 __device__ __forceinline__ uint32_t cluster_rank() {
   uint32_t r;
   asm volatile("mov.u32 %0, %%cluster_ctarank;" : "=r"(r));
+  return r;
+}
+__device__ __forceinline__ uint32_t map_to_rank(uint32_t addr, uint32_t rank) {
+  uint32_t r;
+  asm volatile("mapa.shared::cluster.u32 %0, %1, %2;" : "=r"(r) : "r"(addr), "r"(rank));
   return r;
 }
 __device__ __forceinline__ uint32_t map_to_rank0(uint32_t addr) {
@@ -809,6 +881,21 @@ __device__ __forceinline__ void mma_bf16_cg2(uint32_t d_tmem, uint64_t a, uint64
       "tcgen05.mma.cta_group::2.kind::f16 [%0], %1, %2, %3, p;\n\t}" ::"r"(d_tmem),
       "l"(a), "l"(b), "r"(idesc), "r"(acc));
 }
+// commit to the barrier at `bar`'s offset in every CTA of `mask` (cluster ranks)
+__device__ __forceinline__ void mma_commit_cg2_mask(uint32_t bar, uint16_t mask) {
+  asm volatile("tcgen05.commit.cta_group::2.mbarrier::arrive::one.shared::cluster.multicast::cluster.b64 [%0], %1;" ::"r"(bar),
+               "h"(mask)
+               : "memory");
+}
+// B piece multicast to the CTAs of `mask`; with cta_group::2 the complete_tx of every
+// destination lands on the barrier at bar's offset in that destination's pair leader
+__device__ __forceinline__ void tma_load_2d_cg2_mc(uint32_t dst, const CUtensorMap* map, uint32_t bar_cluster, int c0, int c1,
+                                                   uint16_t mask) {
+  asm volatile(
+      "cp.async.bulk.tensor.2d.cta_group::2.shared::cluster.global.mbarrier::complete_tx::bytes.multicast::cluster [%0], [%1, {%3, %4}], [%2], %5;" ::"r"(dst),
+      "l"((uint64_t)map), "r"(bar_cluster), "r"(c0), "r"(c1), "h"(mask)
+      : "memory");
+}
 __device__ __forceinline__ void mma_commit_cg2(uint32_t bar) {
   asm volatile(
       "{\n\t.reg .b16 m;\n\tmov.b16 m, 3;\n\t"
@@ -818,8 +905,13 @@ __device__ __forceinline__ void mma_commit_cg2(uint32_t bar) {
 __device__ __forceinline__ void mbar_arrive_cluster(uint32_t bar_cluster) {
   asm volatile("mbarrier.arrive.shared::cluster.b64 _, [%0];" ::"r"(bar_cluster) : "memory");
 }
-template <bool OUT_ROWMAJOR>
-__global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(THREADS, 1)
+// CL = 2: one CTA pair per cluster.  CL = 4: two pairs (cluster ranks {0,1} and {2,3}) on
+// vertically adjacent 256×256 tiles of one 512×256 super-tile; they share the B tile, each
+// CTA loading half of its B half (8 KB) by TMA multicast into both pairs, so a CTA reads
+// 24 KB instead of 32 KB from L2 per k-block.  Stage slots are freed by the commits of
+// both pairs (empty barriers count 2, commit mask 0xF).
+template <bool OUT_ROWMAJOR, int CL>
+__global__ void __cluster_dims__(CL, 1, 1) __launch_bounds__(THREADS, 1)
     gemm2_kernel(const __grid_constant__ CUtensorMap mapA, const __grid_constant__ CUtensorMap mapB,
                  const __grid_constant__ Params P) {
   extern __shared__ __align__(1024) uint8_t smem_raw[];
@@ -829,19 +921,23 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(THREADS, 1)
   uint64_t* bars = (uint64_t*)(smem + S2 * STAGE2_BYTES);
   uint32_t* tmem_slot = (uint32_t*)(bars + 2 * S2 + 4);
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
-  const uint32_t rank = cluster_rank();
+  const uint32_t crank = cluster_rank();
+  const uint32_t pp = crank >> 1;                // pair within the cluster
+  const uint32_t rank = crank & 1;               // CTA within the pair
   const bool leader = rank == 0;
+  constexpr int NPP = CL / 2;                    // pairs per cluster
   const uint32_t full0 = smem_u32(bars), empty0 = smem_u32(bars + S2);
   const uint32_t tfull0 = smem_u32(bars + 2 * S2), tempty0 = smem_u32(bars + 2 * S2 + 2);
   // pair tiles: tiles_m/tiles_n count 256×256 tiles; clusters stride over them
-  const int cluster_id = blockIdx.x >> 1, nclusters = gridDim.x >> 1;
+  const int cluster_id = blockIdx.x / CL, nclusters = gridDim.x / CL;
+  const int pair_gid = cluster_id * NPP + (int)pp;   // partial slot / trace row of this pair
 
   if (warp == 0 && lane == 0) {
     asm volatile("prefetch.tensormap [%0];" ::"l"((uint64_t)&mapA) : "memory");
     asm volatile("prefetch.tensormap [%0];" ::"l"((uint64_t)&mapB) : "memory");
     for (int s = 0; s < S2; ++s) {
       mbar_init(full0 + 8 * s, 2);
-      mbar_init(empty0 + 8 * s, 1);
+      mbar_init(empty0 + 8 * s, NPP);
     }
     for (int a = 0; a < 2; ++a) {
       mbar_init(tfull0 + 8 * a, 1);
@@ -865,13 +961,14 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(THREADS, 1)
       // ===== TMA producer (both CTAs; bytes are counted at the leader's full barrier) =====
       int stage = 0;
       uint32_t phase = 0;
-      for (int u = cluster_id; u < P.nunits; u += nclusters) {
-        int t, kb0, kb1, slot;
-        unit_decode(P, u, &t, &kb0, &kb1, &slot);
-        const int m0 = (t / P.tiles_n) * 256 + (int)rank * 128, n0 = (t % P.tiles_n) * 256 + (int)rank * 128;
+      SkIter wi(P, cluster_id, nclusters);
+      SkWork w;
+      while (wi.next(&w)) {
+        const int t = w.t, kb0 = w.kb0, kb1 = w.kb1;
+        const int m0 = ((t / P.tiles_n) * NPP + (int)pp) * 256 + (int)rank * 128, n0 = (t % P.tiles_n) * 256 + (int)rank * 128;
         for (int kb = kb0; kb < kb1; ++kb) {
           mbar_wait(empty0 + 8 * stage, phase ^ 1);
-          const uint32_t fb_leader = map_to_rank0(full0 + 8 * stage);
+          const uint32_t fb_leader = map_to_rank(full0 + 8 * stage, 2 * pp);
           if (leader) mbar_expect_tx(full0 + 8 * stage, 2 * STAGE2_BYTES);
           else mbar_arrive_cluster(fb_leader);
           const uint32_t a_dst = smem_u32(sA + stage * A2_BYTES), b_dst = smem_u32(sB + stage * B2_BYTES);
@@ -887,7 +984,11 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(THREADS, 1)
           } else {
             tma_load_2d_cg2(a_dst, &mapA, fb_leader, k0, m0);
           }
-          if (P.b_mn_major) {
+          if (CL == 4) {               // this pair's 64-row piece of the B half, to both pairs
+            const uint16_t mask = (uint16_t)((1u << rank) | (1u << (2 + rank)));
+            if (P.b_mn_major) tma_load_2d_cg2_mc(b_dst + pp * 8192, &mapB, fb_leader, n0 + 64 * pp, k0, mask);
+            else tma_load_2d_cg2_mc(b_dst + pp * 8192, &mapB, fb_leader, k0, n0 + 64 * pp, mask);
+          } else if (P.b_mn_major) {
             tma_load_2d_cg2(b_dst, &mapB, fb_leader, n0, k0);
             tma_load_2d_cg2(b_dst + 8192, &mapB, fb_leader, n0 + 64, k0);
           } else {
@@ -903,16 +1004,32 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(THREADS, 1)
       int stage = 0;
       uint32_t phase = 0;
       int it = 0;
-      for (int u = cluster_id; u < P.nunits; u += nclusters, ++it) {
-        int t, kb0, kb1, slot;
-        unit_decode(P, u, &t, &kb0, &kb1, &slot);
+      SkIter wi(P, cluster_id, nclusters);
+      SkWork w;
+      for (; wi.next(&w); ++it) {
+        const int u = it;
+        const int kb0 = w.kb0, kb1 = w.kb1;
         const int acc = it & 1;
+        const long long ct0 = P.trace ? clock64() : 0;
         mbar_wait(tempty0 + 8 * acc, ((it >> 1) & 1) ^ 1);
+        if (P.trace && pair_gid + u * nclusters * NPP < P.trace_n)
+          P.trace[8 * (pair_gid + u * nclusters * NPP) + 5] = (unsigned long long)(clock64() - ct0);
         tc_fence_after();
         const uint32_t d = tmem + acc * BN;
+        long long wfull = 0;
         for (int kb = kb0; kb < kb1; ++kb) {
-          mbar_wait(full0 + 8 * stage, phase);
+          if (P.trace) {
+            const long long c0 = clock64();
+            mbar_wait(full0 + 8 * stage, phase);
+            wfull += clock64() - c0;
+          } else {
+            mbar_wait(full0 + 8 * stage, phase);
+          }
           tc_fence_after();
+          if (P.trace && kb == kb0 && pair_gid + u * nclusters * NPP < P.trace_n) {
+            P.trace[8 * (pair_gid + u * nclusters * NPP)] = ((unsigned long long)smid() << 32) | (unsigned)pair_gid;
+            P.trace[8 * (pair_gid + u * nclusters * NPP) + 1] = gtimer();
+          }
           const uint32_t a0 = smem_u32(sA + stage * A2_BYTES), b0 = smem_u32(sB + stage * B2_BYTES);
 #pragma unroll
           for (int k = 0; k < BK / 16; ++k) {
@@ -920,10 +1037,15 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(THREADS, 1)
             const uint64_t bd = P.b_mn_major ? sdesc(b0 + 2048 * k, 8192, 1024) : sdesc(b0 + 32 * k, 16, 1024);
             mma_bf16_cg2(d, ad, bd, P.idesc, (kb != kb0) || k != 0);
           }
-          mma_commit_cg2(empty0 + 8 * stage);
+          if (CL == 4) mma_commit_cg2_mask(empty0 + 8 * stage, 0xF);
+          else mma_commit_cg2(empty0 + 8 * stage);
           if (++stage == S2) { stage = 0; phase ^= 1; }
         }
-        mma_commit_cg2(tfull0 + 8 * acc);
+        mma_commit_cg2_mask(tfull0 + 8 * acc, (uint16_t)(3u << (2 * pp)));
+        if (P.trace && pair_gid + u * nclusters * NPP < P.trace_n) {
+          P.trace[8 * (pair_gid + u * nclusters * NPP) + 2] = gtimer();
+          P.trace[8 * (pair_gid + u * nclusters * NPP) + 4] = (unsigned long long)wfull;
+        }
       }
       // drain: the last accumulators must be released before the barriers go away
       for (int k = 0; k < 2 && it - 1 - k >= 0; ++k) {
@@ -936,31 +1058,31 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(THREADS, 1)
     const int quad = warp & 3;
     const int half = (warp - 2) >> 2;
     const int row = quad * 32 + lane;
-    const uint32_t tempty_leader = map_to_rank0(tempty0);
+    const int ew = rank * 8 + (warp - 2);          // this warp's slot in a stream-K partial
+    const uint32_t stg = smem_u32(smem + S2 * STAGE2_BYTES + 256) + (warp - 2) * 4096;
+    const uint32_t tempty_leader = map_to_rank(tempty0, 2 * pp);
     int it = 0;
-    for (int u = cluster_id; u < P.nunits; u += nclusters, ++it) {
-      int t, kb0, kb1, slot;
-      unit_decode(P, u, &t, &kb0, &kb1, &slot);
+    SkIter wi(P, cluster_id, nclusters);
+    SkWork w;
+    for (; wi.next(&w); ++it) {
+      const int t = w.t;
       const int acc = it & 1;
-      const int64_t m = (int64_t)(t / P.tiles_n) * 256 + rank * 128 + row;
+      const int64_t m = ((int64_t)(t / P.tiles_n) * NPP + pp) * 256 + rank * 128 + row;
       const int64_t n0 = (int64_t)(t % P.tiles_n) * 256 + half * 128;
       mbar_wait(tfull0 + 8 * acc, (it >> 1) & 1);
       tc_fence_after();
       const bool mok = m < P.M;
       const int64_t crow = P.cbase + (OUT_ROWMAJOR ? (mok ? m : 0) * P.ldc : __ldg(P.cM + (mok ? m : 0)));
-      // split-K tail: splits 0..S-2 write a dense fp32 partial tile [256][256] (row =
-      // rank·128 + row) to the workspace and count themselves in at the tile's counter; the
-      // last split (all split units run in the same, final wave) waits for them and folds
-      // p_0 + p_1 + … + own in split order before writing the output
-      const bool split = slot >= 0;
-      const int sidx = split ? slot % P.ssplit : 0, ti = split ? slot / P.ssplit : 0;
-      const bool last = split && sidx == P.ssplit - 1;
-      unsigned* cnt = P.tail_cnt + 2 * ti;
-      const int64_t prel = (int64_t)(rank * 128 + row) * 256 + half * 128;
-      float* prow = (split && !last) ? P.part + (int64_t)slot * 65536 + prel : nullptr;
-      if (last) {
+      // stream-K partials: warp ew of a pair's slot holds its 32 rows × 128 columns as
+      // float4 [c][j][lane] (each store / load instruction covers 512 contiguous bytes)
+      float4* mine = reinterpret_cast<float4*>(P.skpart + (int64_t)pair_gid * 65536 + ew * 4096) + lane;
+      int q1 = cluster_id;                           // finisher: partials of pairs cluster_id+1 .. q1
+      if (w.role == 2) {
+        const int64_t tend = (int64_t)(t - P.nfull + 1) * P.num_kb;
+        while (q1 + 1 < P.sk_pairs && (int64_t)(q1 + 1) * P.sk_w / P.sk_pairs < tend) ++q1;
         if (lane == 0)
-          while (*((volatile unsigned*)cnt) < 16u * (unsigned)(P.ssplit - 1)) __nanosleep(64);
+          for (int q = cluster_id + 1; q <= q1; ++q)
+            while (*((volatile unsigned*)(P.skflag + (q * NPP + pp) * 16 + ew)) == 0u) __nanosleep(64);
         __syncwarp();
         __threadfence();
       }
@@ -969,27 +1091,56 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(THREADS, 1)
         uint32_t r[32];
         tmem_ld32(tmem + ((uint32_t)(quad * 32) << 16) + acc * BN + half * 128 + c * 32, r);
         const int64_t nb = n0 + c * 32;
-        if (last) {
-          const float* p0 = P.part + (int64_t)(ti * P.ssplit) * 65536 + prel + c * 32;
-#pragma unroll
-          for (int j4 = 0; j4 < 8; ++j4) {
-            float4 a = *reinterpret_cast<const float4*>(p0 + 4 * j4);
-            for (int s2 = 1; s2 < P.ssplit - 1; ++s2) {
-              const float4 b = *reinterpret_cast<const float4*>(p0 + (int64_t)s2 * 65536 + 4 * j4);
-              a.x += b.x; a.y += b.y; a.z += b.z; a.w += b.w;
-            }
-            r[4 * j4] = __float_as_uint(a.x + __uint_as_float(r[4 * j4]));
-            r[4 * j4 + 1] = __float_as_uint(a.y + __uint_as_float(r[4 * j4 + 1]));
-            r[4 * j4 + 2] = __float_as_uint(a.z + __uint_as_float(r[4 * j4 + 2]));
-            r[4 * j4 + 3] = __float_as_uint(a.w + __uint_as_float(r[4 * j4 + 3]));
-          }
-        }
-        if (prow) {
-          float4* dst = reinterpret_cast<float4*>(prow + c * 32);
+        if (w.role == 1) {
 #pragma unroll
           for (int j = 0; j < 8; ++j)
-            dst[j] = make_float4(__uint_as_float(r[4 * j]), __uint_as_float(r[4 * j + 1]), __uint_as_float(r[4 * j + 2]),
-                                 __uint_as_float(r[4 * j + 3]));
+            mine[(c * 8 + j) * 32] = make_float4(__uint_as_float(r[4 * j]), __uint_as_float(r[4 * j + 1]),
+                                                 __uint_as_float(r[4 * j + 2]), __uint_as_float(r[4 * j + 3]));
+          continue;
+        }
+        for (int q = cluster_id + 1; q <= q1; ++q) {
+          const float4* src = reinterpret_cast<const float4*>(P.skpart + (int64_t)(q * NPP + pp) * 65536 + ew * 4096) + lane;
+#pragma unroll
+          for (int j = 0; j < 8; ++j) {
+            const float4 b = __ldcg(src + (c * 8 + j) * 32);
+            r[4 * j] = __float_as_uint(__uint_as_float(r[4 * j]) + b.x);
+            r[4 * j + 1] = __float_as_uint(__uint_as_float(r[4 * j + 1]) + b.y);
+            r[4 * j + 2] = __float_as_uint(__uint_as_float(r[4 * j + 2]) + b.z);
+            r[4 * j + 3] = __float_as_uint(__uint_as_float(r[4 * j + 3]) + b.w);
+          }
+        }
+        if (OUT_ROWMAJOR && P.c_vec4) {
+          // transpose through this warp's swizzled 32×32 staging tile (16-byte chunk j of row
+          // r at (j ^ (r & 7))·16: conflict-free both ways), then 8 stores in which 8 lanes
+          // cover one 128-byte row segment, i.e. 4 whole lines per instruction
+#pragma unroll
+          for (int j = 0; j < 8; ++j)
+            asm volatile("st.shared.v4.b32 [%0], {%1, %2, %3, %4};" ::"r"(stg + lane * 128 + ((j ^ (lane & 7)) << 4)),
+                         "r"(r[4 * j]), "r"(r[4 * j + 1]), "r"(r[4 * j + 2]), "r"(r[4 * j + 3])
+                         : "memory");
+          __syncwarp();
+          const int cj = lane & 7;
+          const int64_t ncol = nb + 4 * cj;
+#pragma unroll
+          for (int i = 0; i < 8; ++i) {
+            const int rr = 4 * i + (lane >> 3);
+            const int64_t mm = m - row + quad * 32 + rr;     // this CTA's row quad*32 + rr
+            float4 v;
+            asm volatile("ld.shared.v4.f32 {%0, %1, %2, %3}, [%4];"
+                         : "=f"(v.x), "=f"(v.y), "=f"(v.z), "=f"(v.w)
+                         : "r"(stg + rr * 128 + ((cj ^ (rr & 7)) << 4)));
+            if (mm < P.M) {
+              float* dst = P.C + P.cbase + mm * P.ldc + ncol;
+              if (ncol + 4 <= P.N) {
+                *reinterpret_cast<float4*>(dst) = v;
+              } else {
+                if (ncol < P.N) dst[0] = v.x;
+                if (ncol + 1 < P.N) dst[1] = v.y;
+                if (ncol + 2 < P.N) dst[2] = v.z;
+              }
+            }
+          }
+          __syncwarp();
         } else if (OUT_ROWMAJOR && mok && nb + 32 <= P.N && ((crow + nb) & 3) == 0) {
           float4* dst = reinterpret_cast<float4*>(P.C + crow + nb);
 #pragma unroll
@@ -1002,20 +1153,18 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(THREADS, 1)
             if (nb + j < P.N) P.C[crow + (OUT_ROWMAJOR ? nb + j : __ldg(P.cN + nb + j))] = __uint_as_float(r[j]);
         }
       }
-      if (split && !last) {            // publish this warp's part of the partial tile
+      if (w.role == 1) {               // publish this warp's part of the partial tile
         __threadfence();
         __syncwarp();
-        if (lane == 0) atomicAdd(cnt, 1u);
-      } else if (last) {               // 16 warps (2 CTAs × 8) leave; the last one resets
-        __syncwarp();
-        if (lane == 0 && atomicAdd(cnt + 1, 1u) == 15u) {
-          cnt[0] = 0u;
-          cnt[1] = 0u;
-        }
+        if (lane == 0) atomicExch(P.skflag + pair_gid * 16 + ew, 1u);
+      } else if (w.role == 2 && lane == 0) {
+        for (int q = cluster_id + 1; q <= q1; ++q) P.skflag[(q * NPP + pp) * 16 + ew] = 0u;   // consumed: back to rest
       }
       tc_fence_before();
       __syncwarp();
       if (lane == 0) mbar_arrive_cluster(tempty_leader + 8 * acc);
+      if (P.trace && leader && warp == 2 && lane == 0 && pair_gid + it * nclusters * NPP < P.trace_n)
+        P.trace[8 * (pair_gid + it * nclusters * NPP) + 3] = gtimer();
     }
   }
   __syncwarp();                  // lanes 1..31 of warps 0/1 wait for their role lane
@@ -1027,24 +1176,8 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(THREADS, 1)
   }
 }
 
-// fold the split-K partial tiles of the tail in split order and write them through out_view
-__global__ void __launch_bounds__(256) tail_combine_kernel(const __grid_constant__ Params P) {
-  const int ntail = (P.nunits - P.nfull) / P.ssplit;
-  const int64_t total = (int64_t)ntail * 65536;
-  for (int64_t e = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; e < total; e += (int64_t)gridDim.x * blockDim.x) {
-    const int i = (int)(e >> 16), rc = (int)(e & 65535), r = rc >> 8, c = rc & 255;
-    const int t = P.nfull + i;
-    const int64_t m = (int64_t)(t / P.tiles_n) * 256 + r, n = (int64_t)(t % P.tiles_n) * 256 + c;
-    if (m >= P.M || n >= P.N) continue;
-    const float* src = P.part + (int64_t)i * P.ssplit * 65536 + rc;
-    float acc = src[0];
-    for (int s = 1; s < P.ssplit; ++s) acc += src[(int64_t)s * 65536];
-    const int64_t o = P.cbase + (P.c_rowmajor ? m * P.ldc + n : P.cM[m] + P.cN[n]);
-    P.C[o] = acc;
-  }
-}
-
-constexpr int MAX_TAIL_UNITS = 74;   // partial tiles reserved in the workspace (2-SM path)
+constexpr int SK_MAX_PAIRS = 74;     // stream-K partial slots reserved in the workspace (2-SM path)
+constexpr int SK_MIN_SEG = 8;        // shortest stream-K range per pair, in 64-deep k-blocks
 constexpr int MAX_TAIL_UNITS1 = 296; // 1-SM path: bound on tail units (partials sized per plan)
 
 // ---- operand normalisation pre-pass ---------------------------------------------------
@@ -1228,6 +1361,7 @@ struct T4State {
   t4::Layout2D a, b;
   t4::Params P;
   int cg = 1;      // 1: one SM per 128×256 tile; 2: SM pair per 256×256 tile
+  int cl = 2;      // 2-SM kernel: CTAs per cluster (4: two pairs share B by multicast)
   bool ag = false; // A staged by the kernel's gather warps (no A tensor map, no pre-pass)
   bool ic = false;  // A through a TMA im2col map
   uint64_t ic_dims[4];
@@ -1466,10 +1600,19 @@ mdh_status prepare_t4(Plan* p) {
     P.tiles_n = (int)((c.N + 255) / 256);
     P.num_tiles = P.tiles_m * P.tiles_n;
     P.idesc = (P.idesc & ~(0x1Fu << 24)) | ((uint32_t)(256 >> 4) << 24);
-    // room for the split-K tail's partial tiles (decided at launch from the SM count)
+    // 4-CTA clusters (two pairs on a 512×256 super-tile sharing B; cuBLAS's 4096³ kernel is
+    // 2cta with a 2×2 cluster): L2→SM operand traffic per k-block 24 instead of 32 KB per
+    // CTA.  Opt-in (tile knob cluster=4): only 33 four-CTA clusters are co-resident on a
+    // B200 (132 SMs), and the ~4 % faster k-block rate measured does not pay for the 16 idle
+    // SMs (MatMul 4096³ 120.8 vs 110.7 µs, MCC conv5_1 74.5 vs 68.4 µs).
+    if (P.tiles_m >= 2 && p->tiles.cluster == 4) {
+      s->cl = 4;
+      P.num_tiles = ((P.tiles_m + 1) / 2) * P.tiles_n;
+    }
+    // room for the stream-K partial tiles and flags (decided at launch from the SM count)
     ws = (ws + 255) / 256 * 256;
     s->tail_off = ws;
-    ws += (size_t)t4::MAX_TAIL_UNITS * 65536 * sizeof(float) + 2 * t4::MAX_TAIL_UNITS * sizeof(unsigned) + 256;
+    ws += (size_t)t4::SK_MAX_PAIRS * 65536 * sizeof(float) + 16 * t4::SK_MAX_PAIRS * sizeof(unsigned) + 256;
   } else {
     // 1-SM split-K tail: the T mod C tiles of the last, partial wave split along K over
     // the idle SMs (S units each) — tile knob split=S, or automatically when the partial
@@ -1546,7 +1689,7 @@ mdh_status prepare_t4(Plan* p) {
   p->tiles.bn = s->epi == 3 ? P.bn : t4::BN;
   p->tiles.bk = t4::BK;
   p->tiles.stages = s->cg == 2 ? t4::S2 : (s->epi == 3 ? 2 : t4::STAGES);
-  p->tiles.cluster = s->cg;
+  p->tiles.cluster = s->cg == 2 ? s->cl : 1;
   return MDH_OK;
 }
 
@@ -1600,6 +1743,27 @@ static mdh_status make_im2col_map(CUtensorMap* map, const void* base, const T4St
                   CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
   if (r != CUDA_SUCCESS) { set_error("cuTensorMapEncodeIm2col failed (%d)", (int)r); return MDH_ERR_CUDA; }
   return MDH_OK;
+}
+
+// diagnostics (MDH_T4_TRACE=1): a device buffer for the per-unit timeline of the last
+// 2-SM launch, read back by mdh_debug_t4_trace
+static unsigned long long* g_trace = nullptr;
+static int g_trace_units = 0;
+static unsigned long long* t4_trace_buffer(int units) {
+  static const bool on = std::getenv("MDH_T4_TRACE") && std::getenv("MDH_T4_TRACE")[0] == '1';
+  if (!on) return nullptr;
+  if (units > g_trace_units) {
+    if (g_trace) cudaFree(g_trace);
+    if (cudaMalloc(&g_trace, (size_t)units * 8 * sizeof(unsigned long long)) != cudaSuccess) {
+      cudaGetLastError();
+      g_trace = nullptr;
+      g_trace_units = 0;
+      return nullptr;
+    }
+    g_trace_units = units;
+  }
+  cudaMemset(g_trace, 0, (size_t)g_trace_units * 8 * sizeof(unsigned long long));
+  return g_trace;
 }
 
 // 2-D bf16 tensor map: inner dim `inner` (unit stride), outer dim `outer` with stride ld
@@ -1693,7 +1857,7 @@ mdh_status launch_t4(const Plan& p, const void* const* in, void* const* out, voi
   } else if (s->a.mn_major) MDH_TRY(make_map(&ma, A, c.M, c.K, s->a.ld, 64, 64));
   else MDH_TRY(make_map(&ma, A, c.K, c.M, s->a.ld, 64, 128));
   if (s->b.mn_major) MDH_TRY(make_map(&mb, B, c.N, c.K, s->b.ld, 64, 64));
-  else MDH_TRY(make_map(&mb, B, c.K, c.N, s->b.ld, 64, s->cg == 2 ? 128 : (uint32_t)P.bn));
+  else MDH_TRY(make_map(&mb, B, c.K, c.N, s->b.ld, 64, s->cg == 2 ? (s->cl == 4 ? 64 : 128) : (uint32_t)P.bn));
   if (s->ag) ma = mb;
   static std::once_flag attr_once;
   static cudaError_t attr_err = cudaSuccess;
@@ -1717,7 +1881,8 @@ mdh_status launch_t4(const Plan& p, const void* const* in, void* const* out, voi
                                            (int)(t4::SMEM_LIMIT - t4::BN * sizeof(int64_t)));
       if (e != cudaSuccess) attr_err = e;
     }
-    const void* k2[2] = {(const void*)t4::gemm2_kernel<true>, (const void*)t4::gemm2_kernel<false>};
+    const void* k2[4] = {(const void*)t4::gemm2_kernel<true, 2>, (const void*)t4::gemm2_kernel<false, 2>,
+                         (const void*)t4::gemm2_kernel<true, 4>, (const void*)t4::gemm2_kernel<false, 4>};
     for (const void* k : k2) {
       cudaError_t e = cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, t4::SMEM2_BYTES);
       if (e != cudaSuccess) attr_err = e;
@@ -1729,27 +1894,61 @@ mdh_status launch_t4(const Plan& p, const void* const* in, void* const* out, voi
   cudaGetDevice(&dev);
   cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
   if (s->cg == 2) {
-    // optional split-K tail (tile knob split=S ≥ 2): whole tiles for the complete waves, the
-    // last partial wave's tiles split along K over the idle SM pairs.  Off by default: on
-    // MatMul 4096³ and MCC conv5_1 it measured slower than whole tiles.
-    const int C = std::max(1, std::min(P.num_tiles, sms / 2));
-    const int T = P.num_tiles, R = T / C, Tr = T - R * C;
-    int S = 1;
-    if (Tr > 0 && p.tiles.split > 1) S = std::min({p.tiles.split, C / Tr, t4::MAX_TAIL_UNITS / Tr, P.num_kb});
-    if (S >= 2) {
-      P.nfull = T - Tr;
-      P.ssplit = S;
-      P.nunits = P.nfull + Tr * S;
-      P.part = (float*)((char*)ws + s->tail_off);
-      P.tail_cnt = (unsigned*)((char*)ws + s->tail_off + (size_t)t4::MAX_TAIL_UNITS * 65536 * sizeof(float));
-    } else {
-      P.nfull = T;
-      P.ssplit = 1;
-      P.nunits = T;
-      P.part = nullptr;
+    // stream-K hybrid: with T pair-tiles on C pairs and T mod C ≠ 0, the
+    // first ⌊T/C⌋−1 waves run whole tiles and the rest of the (tile, k-block) space is split
+    // evenly over the pairs (segments of at least SK_MIN_SEG k-blocks); tile knob split=1
+    // keeps whole tiles only
+    const int CL = s->cl, NPP = CL / 2;
+    // the persistent grid must be co-resident (stream-K finishers wait on other clusters):
+    // at most the number of CL-CTA clusters the GPCs can hold at once (for CL = 4 fewer
+    // than sms/4 when a GPC's SM count is not a multiple of 4)
+    static int max_clusters[5] = {0, 0, 0, 0, 0};
+    if (max_clusters[CL] == 0) {
+      cudaLaunchConfig_t cfg = {};
+      cudaLaunchAttribute attr[1];
+      cfg.gridDim = dim3(CL * (sms / CL), 1, 1);
+      cfg.blockDim = dim3(t4::THREADS, 1, 1);
+      cfg.dynamicSmemBytes = t4::SMEM2_BYTES;
+      attr[0].id = cudaLaunchAttributeClusterDimension;
+      attr[0].val.clusterDim.x = CL;
+      attr[0].val.clusterDim.y = 1;
+      attr[0].val.clusterDim.z = 1;
+      cfg.attrs = attr;
+      cfg.numAttrs = 1;
+      int n = 0;
+      const cudaError_t e = CL == 4 ? cudaOccupancyMaxActiveClusters(&n, (const void*)t4::gemm2_kernel<true, 4>, &cfg)
+                                    : cudaOccupancyMaxActiveClusters(&n, (const void*)t4::gemm2_kernel<true, 2>, &cfg);
+      if (e != cudaSuccess || n <= 0) {
+        cudaGetLastError();
+        n = sms / CL;
+      }
+      max_clusters[CL] = std::min(n, sms / CL);
+      if (std::getenv("MDH_T4_TRACE")) fprintf(stderr, "[t4] CL=%d: %d co-resident clusters (occupancy query %d)\n", CL, max_clusters[CL], (int)e);
     }
-    const int grid2 = 2 * std::max(1, std::min(P.nunits, sms / 2));
-    t4::gemm2_kernel<true><<<grid2, t4::THREADS, t4::SMEM2_BYTES, st>>>(ma, mb, P);
+    const int C = std::max(1, max_clusters[CL]);
+    const int T = P.num_tiles, R = T / C;
+    P.nfull = T;
+    P.sk_pairs = 0;
+    P.sk_w = 0;
+    if (T % C != 0 && p.tiles.split != 1) {
+      const int nfull = R >= 1 ? (R - 1) * C : 0;
+      const int64_t W = (int64_t)(T - nfull) * P.num_kb;
+      const int sp = (int)std::min<int64_t>(std::min(C, t4::SK_MAX_PAIRS / NPP), W / t4::SK_MIN_SEG);
+      if (sp >= 2) {
+        P.nfull = nfull;
+        P.sk_pairs = sp;
+        P.sk_w = W;
+        P.skpart = (float*)((char*)ws + s->tail_off);
+        P.skflag = (unsigned*)((char*)ws + s->tail_off + (size_t)t4::SK_MAX_PAIRS * 65536 * sizeof(float));
+      }
+    }
+    const int clusters = P.sk_pairs > 0 ? C : std::max(1, std::min(T, C));
+    P.trace = t4_trace_buffer(clusters * NPP * (T / clusters + 4));
+    P.trace_n = P.trace ? clusters * NPP * (T / clusters + 4) : 0;
+    const int grid2 = CL * clusters;
+    P.c_vec4 = P.c_rowmajor && P.ldc % 4 == 0 && P.cbase % 4 == 0 && (uintptr_t)P.C % 16 == 0;
+    if (CL == 4) t4::gemm2_kernel<true, 4><<<grid2, t4::THREADS, t4::SMEM2_BYTES, st>>>(ma, mb, P);
+    else t4::gemm2_kernel<true, 2><<<grid2, t4::THREADS, t4::SMEM2_BYTES, st>>>(ma, mb, P);
     return post_launch("t4_gemm2_kernel");
   }
   int grid = std::min(P.num_tiles, sms);
@@ -1787,3 +1986,14 @@ mdh_status launch_t4(const Plan& p, const void* const* in, void* const* out, voi
 }
 
 }  // namespace mdh
+
+extern "C" int64_t mdh_debug_t4_trace(uint64_t* host, int64_t max_units) {
+  if (!mdh::g_trace || !host) return 0;
+  const int64_t n = std::min<int64_t>(max_units, mdh::g_trace_units);
+  if (cudaDeviceSynchronize() != cudaSuccess ||
+      cudaMemcpy(host, mdh::g_trace, (size_t)n * 8 * sizeof(uint64_t), cudaMemcpyDeviceToHost) != cudaSuccess) {
+    cudaGetLastError();
+    return -1;
+  }
+  return n;
+}

@@ -93,6 +93,8 @@ def lib():
             L.mdh_last_error.restype = ctypes.c_char_p
             L.mdh_abi_version.restype = ctypes.c_int32
             L.mdh_last_launch_count.restype = ctypes.c_int32
+            L.mdh_debug_t4_trace.argtypes = [P, ctypes.c_int64]
+            L.mdh_debug_t4_trace.restype = ctypes.c_int64
             for name in ("mdh_plan", "mdh_plan_workspace_size", "mdh_plan_local_shape", "mdh_plan_describe",
                          "mdh_execute", "mdh_plan_host_scratch_size", "mdh_execute_host",
                          "mdh_combine_partials", "mdh_destroy", "mdh_comm_unique_id", "mdh_comm_init",
@@ -281,6 +283,18 @@ class Plan:
     @staticmethod
     def last_launch_count() -> int:
         return int(lib().mdh_last_launch_count())
+
+    @staticmethod
+    def t4_trace(max_units: int = 65536):
+        """Diagnostics: the T4 2-SM per-unit timeline of the last launch (MDH_T4_TRACE=1),
+        as a list of (sm, pair, t_first_mma, t_last_commit, t_epilogue_done) in ns and
+        (wait_full, wait_accumulator) in SM cycles."""
+        buf = (ctypes.c_uint64 * (8 * max_units))()
+        n = int(lib().mdh_debug_t4_trace(buf, max_units))
+        if n < 0:
+            raise MdhError(-1, "mdh_debug_t4_trace failed")
+        return [(buf[8 * u] >> 32, buf[8 * u] & 0xffffffff, buf[8 * u + 1], buf[8 * u + 2], buf[8 * u + 3],
+                 buf[8 * u + 4], buf[8 * u + 5]) for u in range(n) if buf[8 * u + 1]]
 
 
 class Comm:

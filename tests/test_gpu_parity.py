@@ -465,6 +465,41 @@ def test_t4_split_tail_1sm(shape, tile, out):
         assert_close_points(spec, x, got, 1e-2, n=20000, kind="rel")
 
 
+@pytest.mark.parametrize("shape,tile,kind", [((512, 512, 8192), None, "full"),       # 4 tiles, ~16 pairs each
+                                             ((2500, 2000, 1000), None, "points"),   # ragged, 80 tiles / 74 pairs
+                                             ((4096, 4096, 4096), None, "points"),   # 2 data-parallel waves + SK
+                                             ((1024, 768, 640), "split=1", "full"),   # whole tiles only
+                                             ((700, 1000, 1000), "cluster=4", "full"),  # odd row tiles: an idle pair
+                                             ((2500, 2000, 1000), "cluster=4", "points")])  # 4-CTA clusters
+def test_t4_stream_k(shape, tile, kind):
+    """2-SM stream-K hybrid: whole-tile waves, then each cluster's even share of the remaining
+    (tile, k-block) space; producers publish coalesced fp32 partials, the finisher (the one
+    holding k = 0) adds them in k order.  Single pairs (default) and 4-CTA clusters
+    (cluster=4: two pairs sharing B by TMA multicast; with an odd number of 256-row tiles
+    the last pair computes zero-filled rows and stores nothing).  Run twice on one plan:
+    the flags return to rest."""
+    M, N, K = shape
+    spec = S.matmul(M, N, K, "bf16")
+    x = G.matmul_inputs(M, N, K, "bf16", "positive")
+    plan = None
+    first = None
+    for _ in range(2):
+        got, plan = run_gpu(spec, x, plan=plan, force_tile=tile)
+        assert plan.describe()["t4_variant"] & 8
+        if kind == "full":
+            assert_close_full(spec, x, got, 1e-2, kind="rel")
+        else:
+            assert_close_points(spec, x, got, 1e-2, n=20000, kind="rel")
+        if first is None:
+            first = got[0].copy()
+        else:
+            assert np.array_equal(first, got[0])          # deterministic fixup order
+    if shape == (4096, 4096, 4096):
+        ones = G.matmul_inputs(M, N, K, "bf16", "ones")
+        got, _ = run_gpu(spec, ones, plan=plan)
+        assert np.all(got[0] == float(K))
+
+
 def test_mcc_bf16_config_sampled():
     spec = S.mcc(256, 7, 7, 512, 3, 3, 512, "bf16")
     x = G.mcc_inputs(spec)
