@@ -221,7 +221,8 @@ int32_t mdh_last_launch_count(void);
  * the T4 2-SM tensor-core kernel records, per work unit u of its last launch, eight u64 at
  * host[8u..8u+7]: (SM id << 32 | CTA-pair id, %globaltimer ns at the unit's first MMA
  * issue, at its last MMA commit, at the end of its epilogue, SM cycles the MMA issuer
- * waited for loaded stages, SM cycles it waited for a free accumulator, 0, 0).  Synchronises the device,
+ * waited for loaded stages, SM cycles it waited for a free accumulator, %globaltimer when a
+ * stream-K finisher saw all its partials, when a producer published its partial; else 0).  Synchronises the device,
  * copies at most max_units units and returns how many; 0 when tracing is off, -1 on a
  * CUDA error.  `host` is caller-owned.                                                  */
 int64_t mdh_debug_t4_trace(uint64_t* host, int64_t max_units);

@@ -842,7 +842,9 @@ constexpr int A2_BYTES = 128 * BK * 2;         // this CTA's half of A (16 KB)
 constexpr int B2_BYTES = 128 * BK * 2;         // this CTA's half of B (16 KB)
 constexpr int STAGE2_BYTES = A2_BYTES + B2_BYTES;
 constexpr int STG2_BYTES = 8 * 32 * 32 * 4;    // epilogue staging: 32×32 fp32 per epilogue warp
+constexpr int S2W = 4;                         // stages of the wide (NW = 512) ring (48 KB each)
 constexpr int SMEM2_BYTES = S2 * STAGE2_BYTES + 1024 + 256 + STG2_BYTES;
+static_assert(S2W * (A2_BYTES + 2 * B2_BYTES) <= S2 * STAGE2_BYTES, "wide ring must fit the 2-SM smem budget");
 
 __device__ __forceinline__ uint32_t cluster_rank() {
   uint32_t r;
@@ -910,32 +912,42 @@ __device__ __forceinline__ void mbar_arrive_cluster(uint32_t bar_cluster) {
 // CTA loading half of its B half (8 KB) by TMA multicast into both pairs, so a CTA reads
 // 24 KB instead of 32 KB from L2 per k-block.  Stage slots are freed by the commits of
 // both pairs (empty barriers count 2, commit mask 0xF).
-template <bool OUT_ROWMAJOR, int CL>
+//
+// NW = 512 (wide tiles, CL = 2): a pair owns a 256×512 tile as two N=256 MMAs per k-step
+// into TMEM columns [0,256) and [256,512) — all 512 columns, so there is one accumulator:
+// the epilogue drains column half 0, frees it (tempty[0]), then half 1 (tempty[1]), and the
+// next tile's first MMAs into half h wait only for tempty[h].  Per k-block a CTA loads its
+// A half once for twice the MMA work (A 16 + B 32 KB per 8.4 MFLOP instead of 16 + 16 per
+// 4.2): A — the im2col operand of a convolution — is requested half as often.
+template <bool OUT_ROWMAJOR, int CL, int NW = 256>
 __global__ void __cluster_dims__(CL, 1, 1) __launch_bounds__(THREADS, 1)
     gemm2_kernel(const __grid_constant__ CUtensorMap mapA, const __grid_constant__ CUtensorMap mapB,
                  const __grid_constant__ Params P) {
   extern __shared__ __align__(1024) uint8_t smem_raw[];
+  constexpr int NH = NW / 256;                   // N=256 MMAs per k-step
+  constexpr int NS = NW == 512 ? S2W : S2;       // ring stages
+  constexpr int BSTG = NH * B2_BYTES;            // this CTA's B bytes per stage
   uint8_t* smem = (uint8_t*)(((uintptr_t)smem_raw + 1023) & ~(uintptr_t)1023);
   uint8_t* sA = smem;
-  uint8_t* sB = smem + S2 * A2_BYTES;
-  uint64_t* bars = (uint64_t*)(smem + S2 * STAGE2_BYTES);
-  uint32_t* tmem_slot = (uint32_t*)(bars + 2 * S2 + 4);
+  uint8_t* sB = smem + NS * A2_BYTES;
+  uint64_t* bars = (uint64_t*)(smem + NS * (A2_BYTES + BSTG));
+  uint32_t* tmem_slot = (uint32_t*)(bars + 2 * NS + 4);
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const uint32_t crank = cluster_rank();
   const uint32_t pp = crank >> 1;                // pair within the cluster
   const uint32_t rank = crank & 1;               // CTA within the pair
   const bool leader = rank == 0;
   constexpr int NPP = CL / 2;                    // pairs per cluster
-  const uint32_t full0 = smem_u32(bars), empty0 = smem_u32(bars + S2);
-  const uint32_t tfull0 = smem_u32(bars + 2 * S2), tempty0 = smem_u32(bars + 2 * S2 + 2);
-  // pair tiles: tiles_m/tiles_n count 256×256 tiles; clusters stride over them
+  const uint32_t full0 = smem_u32(bars), empty0 = smem_u32(bars + NS);
+  const uint32_t tfull0 = smem_u32(bars + 2 * NS), tempty0 = smem_u32(bars + 2 * NS + 2);
+  // pair tiles: tiles_m/tiles_n count 256×NW tiles; clusters stride over them
   const int cluster_id = blockIdx.x / CL, nclusters = gridDim.x / CL;
   const int pair_gid = cluster_id * NPP + (int)pp;   // partial slot / trace row of this pair
 
   if (warp == 0 && lane == 0) {
     asm volatile("prefetch.tensormap [%0];" ::"l"((uint64_t)&mapA) : "memory");
     asm volatile("prefetch.tensormap [%0];" ::"l"((uint64_t)&mapB) : "memory");
-    for (int s = 0; s < S2; ++s) {
+    for (int s = 0; s < NS; ++s) {
       mbar_init(full0 + 8 * s, 2);
       mbar_init(empty0 + 8 * s, NPP);
     }
@@ -965,13 +977,13 @@ __global__ void __cluster_dims__(CL, 1, 1) __launch_bounds__(THREADS, 1)
       SkWork w;
       while (wi.next(&w)) {
         const int t = w.t, kb0 = w.kb0, kb1 = w.kb1;
-        const int m0 = ((t / P.tiles_n) * NPP + (int)pp) * 256 + (int)rank * 128, n0 = (t % P.tiles_n) * 256 + (int)rank * 128;
+        const int m0 = ((t / P.tiles_n) * NPP + (int)pp) * 256 + (int)rank * 128, n0 = (t % P.tiles_n) * NW + (int)rank * 128;
         for (int kb = kb0; kb < kb1; ++kb) {
           mbar_wait(empty0 + 8 * stage, phase ^ 1);
           const uint32_t fb_leader = map_to_rank(full0 + 8 * stage, 2 * pp);
-          if (leader) mbar_expect_tx(full0 + 8 * stage, 2 * STAGE2_BYTES);
+          if (leader) mbar_expect_tx(full0 + 8 * stage, 2 * (A2_BYTES + BSTG));
           else mbar_arrive_cluster(fb_leader);
-          const uint32_t a_dst = smem_u32(sA + stage * A2_BYTES), b_dst = smem_u32(sB + stage * B2_BYTES);
+          const uint32_t a_dst = smem_u32(sA + stage * A2_BYTES), b_dst = smem_u32(sB + stage * BSTG);
           const int k0 = krotate(P, kb, kb0, kb1, t / P.tiles_n) * BK;
           if (P.a_im2col) {
             int cr[4];
@@ -988,13 +1000,18 @@ __global__ void __cluster_dims__(CL, 1, 1) __launch_bounds__(THREADS, 1)
             const uint16_t mask = (uint16_t)((1u << rank) | (1u << (2 + rank)));
             if (P.b_mn_major) tma_load_2d_cg2_mc(b_dst + pp * 8192, &mapB, fb_leader, n0 + 64 * pp, k0, mask);
             else tma_load_2d_cg2_mc(b_dst + pp * 8192, &mapB, fb_leader, k0, n0 + 64 * pp, mask);
-          } else if (P.b_mn_major) {
-            tma_load_2d_cg2(b_dst, &mapB, fb_leader, n0, k0);
-            tma_load_2d_cg2(b_dst + 8192, &mapB, fb_leader, n0 + 64, k0);
           } else {
-            tma_load_2d_cg2(b_dst, &mapB, fb_leader, k0, n0);
+#pragma unroll
+            for (int h = 0; h < NH; ++h) {   // B piece h: columns 256h + 128·rank + [0, 128)
+              if (P.b_mn_major) {
+                tma_load_2d_cg2(b_dst + h * B2_BYTES, &mapB, fb_leader, n0 + 256 * h, k0);
+                tma_load_2d_cg2(b_dst + h * B2_BYTES + 8192, &mapB, fb_leader, n0 + 256 * h + 64, k0);
+              } else {
+                tma_load_2d_cg2(b_dst + h * B2_BYTES, &mapB, fb_leader, k0, n0 + 256 * h);
+              }
+            }
           }
-          if (++stage == S2) { stage = 0; phase ^= 1; }
+          if (++stage == NS) { stage = 0; phase ^= 1; }
         }
       }
     }
@@ -1009,12 +1026,14 @@ __global__ void __cluster_dims__(CL, 1, 1) __launch_bounds__(THREADS, 1)
       for (; wi.next(&w); ++it) {
         const int u = it;
         const int kb0 = w.kb0, kb1 = w.kb1;
-        const int acc = it & 1;
+        const int acc = NH == 1 ? it & 1 : 0;
         const long long ct0 = P.trace ? clock64() : 0;
-        mbar_wait(tempty0 + 8 * acc, ((it >> 1) & 1) ^ 1);
-        if (P.trace && pair_gid + u * nclusters * NPP < P.trace_n)
-          P.trace[8 * (pair_gid + u * nclusters * NPP) + 5] = (unsigned long long)(clock64() - ct0);
-        tc_fence_after();
+        if (NH == 1) {
+          mbar_wait(tempty0 + 8 * acc, ((it >> 1) & 1) ^ 1);
+          if (P.trace && pair_gid + u * nclusters * NPP < P.trace_n)
+            P.trace[8 * (pair_gid + u * nclusters * NPP) + 5] = (unsigned long long)(clock64() - ct0);
+          tc_fence_after();
+        }
         const uint32_t d = tmem + acc * BN;
         long long wfull = 0;
         for (int kb = kb0; kb < kb1; ++kb) {
@@ -1030,16 +1049,27 @@ __global__ void __cluster_dims__(CL, 1, 1) __launch_bounds__(THREADS, 1)
             P.trace[8 * (pair_gid + u * nclusters * NPP)] = ((unsigned long long)smid() << 32) | (unsigned)pair_gid;
             P.trace[8 * (pair_gid + u * nclusters * NPP) + 1] = gtimer();
           }
-          const uint32_t a0 = smem_u32(sA + stage * A2_BYTES), b0 = smem_u32(sB + stage * B2_BYTES);
+          const uint32_t a0 = smem_u32(sA + stage * A2_BYTES), b0 = smem_u32(sB + stage * BSTG);
 #pragma unroll
-          for (int k = 0; k < BK / 16; ++k) {
-            const uint64_t ad = P.a_mn_major ? sdesc(a0 + 2048 * k, 8192, 1024) : sdesc(a0 + 32 * k, 16, 1024);
-            const uint64_t bd = P.b_mn_major ? sdesc(b0 + 2048 * k, 8192, 1024) : sdesc(b0 + 32 * k, 16, 1024);
-            mma_bf16_cg2(d, ad, bd, P.idesc, (kb != kb0) || k != 0);
+          for (int h = 0; h < NH; ++h) {
+            if (NH > 1 && kb == kb0) {      // column half h of the accumulator drained?
+              const long long ch = P.trace ? clock64() : 0;
+              mbar_wait(tempty0 + 8 * h, (it & 1) ^ 1);
+              if (P.trace && pair_gid + u * nclusters * NPP < P.trace_n)
+                P.trace[8 * (pair_gid + u * nclusters * NPP) + 5] += (unsigned long long)(clock64() - ch);
+              tc_fence_after();
+            }
+#pragma unroll
+            for (int k = 0; k < BK / 16; ++k) {
+              const uint64_t ad = P.a_mn_major ? sdesc(a0 + 2048 * k, 8192, 1024) : sdesc(a0 + 32 * k, 16, 1024);
+              const uint32_t bh = b0 + h * B2_BYTES;
+              const uint64_t bd = P.b_mn_major ? sdesc(bh + 2048 * k, 8192, 1024) : sdesc(bh + 32 * k, 16, 1024);
+              mma_bf16_cg2(d + 256 * h, ad, bd, P.idesc, (kb != kb0) || k != 0);
+            }
           }
           if (CL == 4) mma_commit_cg2_mask(empty0 + 8 * stage, 0xF);
           else mma_commit_cg2(empty0 + 8 * stage);
-          if (++stage == S2) { stage = 0; phase ^= 1; }
+          if (++stage == NS) { stage = 0; phase ^= 1; }
         }
         mma_commit_cg2_mask(tfull0 + 8 * acc, (uint16_t)(3u << (2 * pp)));
         if (P.trace && pair_gid + u * nclusters * NPP < P.trace_n) {
@@ -1048,9 +1078,14 @@ __global__ void __cluster_dims__(CL, 1, 1) __launch_bounds__(THREADS, 1)
         }
       }
       // drain: the last accumulators must be released before the barriers go away
-      for (int k = 0; k < 2 && it - 1 - k >= 0; ++k) {
-        const int j = it - 1 - k;
-        mbar_wait(tempty0 + 8 * (j & 1), (j >> 1) & 1);
+      if (NH == 1) {
+        for (int k = 0; k < 2 && it - 1 - k >= 0; ++k) {
+          const int j = it - 1 - k;
+          mbar_wait(tempty0 + 8 * (j & 1), (j >> 1) & 1);
+        }
+      } else if (it > 0) {
+        mbar_wait(tempty0, (it - 1) & 1);
+        mbar_wait(tempty0 + 8, (it - 1) & 1);
       }
     }
   } else {
@@ -1059,23 +1094,23 @@ __global__ void __cluster_dims__(CL, 1, 1) __launch_bounds__(THREADS, 1)
     const int half = (warp - 2) >> 2;
     const int row = quad * 32 + lane;
     const int ew = rank * 8 + (warp - 2);          // this warp's slot in a stream-K partial
-    const uint32_t stg = smem_u32(smem + S2 * STAGE2_BYTES + 256) + (warp - 2) * 4096;
+    const uint32_t stg = smem_u32(smem + NS * (A2_BYTES + BSTG) + 256) + (warp - 2) * 4096;
     const uint32_t tempty_leader = map_to_rank(tempty0, 2 * pp);
     int it = 0;
     SkIter wi(P, cluster_id, nclusters);
     SkWork w;
     for (; wi.next(&w); ++it) {
       const int t = w.t;
-      const int acc = it & 1;
+      const int acc = NH == 1 ? it & 1 : 0;
       const int64_t m = ((int64_t)(t / P.tiles_n) * NPP + pp) * 256 + rank * 128 + row;
-      const int64_t n0 = (int64_t)(t % P.tiles_n) * 256 + half * 128;
-      mbar_wait(tfull0 + 8 * acc, (it >> 1) & 1);
+      const int64_t ntile = (int64_t)(t % P.tiles_n) * NW;
+      mbar_wait(tfull0 + 8 * acc, NH == 1 ? (it >> 1) & 1 : it & 1);
       tc_fence_after();
       const bool mok = m < P.M;
       const int64_t crow = P.cbase + (OUT_ROWMAJOR ? (mok ? m : 0) * P.ldc : __ldg(P.cM + (mok ? m : 0)));
       // stream-K partials: warp ew of a pair's slot holds its 32 rows × 128 columns as
       // float4 [c][j][lane] (each store / load instruction covers 512 contiguous bytes)
-      float4* mine = reinterpret_cast<float4*>(P.skpart + (int64_t)pair_gid * 65536 + ew * 4096) + lane;
+      float4* mine = reinterpret_cast<float4*>(P.skpart + (int64_t)pair_gid * (NH * 65536) + ew * (NH * 4096)) + lane;
       int q1 = cluster_id;                           // finisher: partials of pairs cluster_id+1 .. q1
       if (w.role == 2) {
         const int64_t tend = (int64_t)(t - P.nfull + 1) * P.num_kb;
@@ -1085,24 +1120,38 @@ __global__ void __cluster_dims__(CL, 1, 1) __launch_bounds__(THREADS, 1)
             while (*((volatile unsigned*)(P.skflag + (q * NPP + pp) * 16 + ew)) == 0u) __nanosleep(64);
         __syncwarp();
         __threadfence();
+        if (P.trace && leader && warp == 2 && lane == 0 && pair_gid + it * nclusters * NPP < P.trace_n)
+          P.trace[8 * (pair_gid + it * nclusters * NPP) + 6] = gtimer();
       }
-#pragma unroll 1
-      for (int c = 0; c < 4; ++c) {
-        uint32_t r[32];
-        tmem_ld32(tmem + ((uint32_t)(quad * 32) << 16) + acc * BN + half * 128 + c * 32, r);
-        const int64_t nb = n0 + c * 32;
-        if (w.role == 1) {
+      auto epi_chunk = [&](uint32_t* r, int64_t nb, int pc) {
+        // fold the producers' partials in k order, two partials' loads in flight at a time
+        // (the fold is latency-bound: 16 independent 512-byte warp loads per round trip)
+        auto part = [&](int q) {
+          return reinterpret_cast<const float4*>(P.skpart + (int64_t)(q * NPP + pp) * (NH * 65536) + ew * (NH * 4096)) +
+                 lane + pc * 8 * 32;
+        };
+        int q = cluster_id + 1;
+        for (; q + 1 <= q1; q += 2) {
+          const float4* s0 = part(q);
+          const float4* s1 = part(q + 1);
+          float4 b0[8], b1[8];
 #pragma unroll
-          for (int j = 0; j < 8; ++j)
-            mine[(c * 8 + j) * 32] = make_float4(__uint_as_float(r[4 * j]), __uint_as_float(r[4 * j + 1]),
-                                                 __uint_as_float(r[4 * j + 2]), __uint_as_float(r[4 * j + 3]));
-          continue;
-        }
-        for (int q = cluster_id + 1; q <= q1; ++q) {
-          const float4* src = reinterpret_cast<const float4*>(P.skpart + (int64_t)(q * NPP + pp) * 65536 + ew * 4096) + lane;
+          for (int j = 0; j < 8; ++j) b0[j] = __ldcg(s0 + j * 32);
+#pragma unroll
+          for (int j = 0; j < 8; ++j) b1[j] = __ldcg(s1 + j * 32);
 #pragma unroll
           for (int j = 0; j < 8; ++j) {
-            const float4 b = __ldcg(src + (c * 8 + j) * 32);
+            r[4 * j] = __float_as_uint(__uint_as_float(r[4 * j]) + b0[j].x + b1[j].x);
+            r[4 * j + 1] = __float_as_uint(__uint_as_float(r[4 * j + 1]) + b0[j].y + b1[j].y);
+            r[4 * j + 2] = __float_as_uint(__uint_as_float(r[4 * j + 2]) + b0[j].z + b1[j].z);
+            r[4 * j + 3] = __float_as_uint(__uint_as_float(r[4 * j + 3]) + b0[j].w + b1[j].w);
+          }
+        }
+        if (q <= q1) {
+          const float4* s0 = part(q);
+#pragma unroll
+          for (int j = 0; j < 8; ++j) {
+            const float4 b = __ldcg(s0 + j * 32);
             r[4 * j] = __float_as_uint(__uint_as_float(r[4 * j]) + b.x);
             r[4 * j + 1] = __float_as_uint(__uint_as_float(r[4 * j + 1]) + b.y);
             r[4 * j + 2] = __float_as_uint(__uint_as_float(r[4 * j + 2]) + b.z);
@@ -1152,17 +1201,49 @@ __global__ void __cluster_dims__(CL, 1, 1) __launch_bounds__(THREADS, 1)
           for (int j = 0; j < 32; ++j)
             if (nb + j < P.N) P.C[crow + (OUT_ROWMAJOR ? nb + j : __ldg(P.cN + nb + j))] = __uint_as_float(r[j]);
         }
+      };
+#pragma unroll 1
+      for (int h = 0; h < NH; ++h) {
+      const int64_t n0 = ntile + 256 * h + half * 128;
+      const uint32_t tb = tmem + ((uint32_t)(quad * 32) << 16) + acc * BN + 256 * h + half * 128;
+      // (a software-pipelined variant — TMEM load of chunk c+1 in flight while chunk c is
+      // stored — measured 1-3 % slower: the epilogue is bound by the memory system, not by
+      // the TMEM load latency)
+#pragma unroll 1
+      for (int c = 0; c < 4; ++c) {
+        uint32_t r[32];
+        tmem_ld32(tb + c * 32, r);
+        const int64_t nb = n0 + c * 32;
+        const int pc = h * 4 + c;                    // 32-column chunk index in the partial
+        if (w.role == 1) {
+#pragma unroll
+          for (int j = 0; j < 8; ++j)
+            mine[(pc * 8 + j) * 32] = make_float4(__uint_as_float(r[4 * j]), __uint_as_float(r[4 * j + 1]),
+                                                  __uint_as_float(r[4 * j + 2]), __uint_as_float(r[4 * j + 3]));
+        } else {
+          epi_chunk(r, nb, pc);
+        }
+      }
+      if (NH > 1) {                    // column half h read out: the next tile may write it
+        tc_fence_before();
+        __syncwarp();
+        if (lane == 0) mbar_arrive_cluster(tempty_leader + 8 * h);
+      }
       }
       if (w.role == 1) {               // publish this warp's part of the partial tile
         __threadfence();
         __syncwarp();
         if (lane == 0) atomicExch(P.skflag + pair_gid * 16 + ew, 1u);
+        if (P.trace && leader && warp == 2 && lane == 0 && pair_gid + it * nclusters * NPP < P.trace_n)
+          P.trace[8 * (pair_gid + it * nclusters * NPP) + 7] = gtimer();
       } else if (w.role == 2 && lane == 0) {
         for (int q = cluster_id + 1; q <= q1; ++q) P.skflag[(q * NPP + pp) * 16 + ew] = 0u;   // consumed: back to rest
       }
-      tc_fence_before();
-      __syncwarp();
-      if (lane == 0) mbar_arrive_cluster(tempty_leader + 8 * acc);
+      if (NH == 1) {
+        tc_fence_before();
+        __syncwarp();
+        if (lane == 0) mbar_arrive_cluster(tempty_leader + 8 * acc);
+      }
       if (P.trace && leader && warp == 2 && lane == 0 && pair_gid + it * nclusters * NPP < P.trace_n)
         P.trace[8 * (pair_gid + it * nclusters * NPP) + 3] = gtimer();
     }
@@ -1362,6 +1443,7 @@ struct T4State {
   t4::Params P;
   int cg = 1;      // 1: one SM per 128×256 tile; 2: SM pair per 256×256 tile
   int cl = 2;      // 2-SM kernel: CTAs per cluster (4: two pairs share B by multicast)
+  int nw = 256;    // 2-SM kernel: N extent of a pair tile (512: two MMAs per k-step)
   bool ag = false; // A staged by the kernel's gather warps (no A tensor map, no pre-pass)
   bool ic = false;  // A through a TMA im2col map
   uint64_t ic_dims[4];
@@ -1377,6 +1459,15 @@ struct T4State {
   uint64_t bdims[5], bstrides[4];
   uint32_t bbox[5];
 };
+
+static int plan_sms(const Plan* p) {
+  int sms = 148;
+  if (cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, p->device) != cudaSuccess || sms <= 0) {
+    cudaGetLastError();
+    sms = 148;
+  }
+  return sms;
+}
 
 // Implicit-GEMM planning for A (e.g. MCC's img[n, 2p+r, 2q+s, c]): pick g* (an M dim with a
 // unit coefficient on one buffer coordinate, extent a multiple of the 128-row tile) and k*
@@ -1608,11 +1699,21 @@ mdh_status prepare_t4(Plan* p) {
     if (P.tiles_m >= 2 && p->tiles.cluster == 4) {
       s->cl = 4;
       P.num_tiles = ((P.tiles_m + 1) / 2) * P.tiles_n;
+    } else if (c.N > 256 && p->tiles.bn != 256 &&
+               (p->tiles.bn == 512 || icp.a_im2col ||
+                (int64_t)P.tiles_m * ((c.N + 511) / 512) >= 2 * std::max(1, plan_sms(p) / 2))) {
+      // wide pair tiles 256×512: A is requested once per 8.4 MFLOP instead of
+      // per 4.2.  Auto for an im2col A (MCC conv5_1: 67.6 vs 71.8 µs) and for GEMMs with at
+      // least two waves of wide tiles (8192³: 1461 vs 1321 TFLOP/s; at 4096³, 1.7 waves, the
+      // narrow tiles' overlapped epilogues win: 114.7 vs 115.7 µs); tile knob bn=256|512
+      s->nw = 512;
+      P.tiles_n = (int)((c.N + 511) / 512);
+      P.num_tiles = P.tiles_m * P.tiles_n;
     }
     // room for the stream-K partial tiles and flags (decided at launch from the SM count)
     ws = (ws + 255) / 256 * 256;
     s->tail_off = ws;
-    ws += (size_t)t4::SK_MAX_PAIRS * 65536 * sizeof(float) + 16 * t4::SK_MAX_PAIRS * sizeof(unsigned) + 256;
+    ws += (size_t)t4::SK_MAX_PAIRS * (s->nw / 256) * 65536 * sizeof(float) + 16 * t4::SK_MAX_PAIRS * sizeof(unsigned) + 256;
   } else {
     // 1-SM split-K tail: the T mod C tiles of the last, partial wave split along K over
     // the idle SMs (S units each) — tile knob split=S, or automatically when the partial
@@ -1686,7 +1787,7 @@ mdh_status prepare_t4(Plan* p) {
                   (a_gather ? 32 : 0) + (s->epi == 2 ? 64 : 0) + (s->epi == 3 ? 128 : 0) + (a_ic ? 256 : 0);
   p->ws_kernel = ws;
   p->tiles.bm = s->cg == 2 ? 256 : t4::BM;
-  p->tiles.bn = s->epi == 3 ? P.bn : t4::BN;
+  p->tiles.bn = s->epi == 3 ? P.bn : (s->cg == 2 ? s->nw : t4::BN);
   p->tiles.bk = t4::BK;
   p->tiles.stages = s->cg == 2 ? t4::S2 : (s->epi == 3 ? 2 : t4::STAGES);
   p->tiles.cluster = s->cg == 2 ? s->cl : 1;
@@ -1881,8 +1982,9 @@ mdh_status launch_t4(const Plan& p, const void* const* in, void* const* out, voi
                                            (int)(t4::SMEM_LIMIT - t4::BN * sizeof(int64_t)));
       if (e != cudaSuccess) attr_err = e;
     }
-    const void* k2[4] = {(const void*)t4::gemm2_kernel<true, 2>, (const void*)t4::gemm2_kernel<false, 2>,
-                         (const void*)t4::gemm2_kernel<true, 4>, (const void*)t4::gemm2_kernel<false, 4>};
+    const void* k2[5] = {(const void*)t4::gemm2_kernel<true, 2>, (const void*)t4::gemm2_kernel<false, 2>,
+                         (const void*)t4::gemm2_kernel<true, 4>, (const void*)t4::gemm2_kernel<false, 4>,
+                         (const void*)t4::gemm2_kernel<true, 2, 512>};
     for (const void* k : k2) {
       cudaError_t e = cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, t4::SMEM2_BYTES);
       if (e != cudaSuccess) attr_err = e;
@@ -1895,9 +1997,9 @@ mdh_status launch_t4(const Plan& p, const void* const* in, void* const* out, voi
   cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
   if (s->cg == 2) {
     // stream-K hybrid: with T pair-tiles on C pairs and T mod C ≠ 0, the
-    // first ⌊T/C⌋−1 waves run whole tiles and the rest of the (tile, k-block) space is split
-    // evenly over the pairs (segments of at least SK_MIN_SEG k-blocks); tile knob split=1
-    // keeps whole tiles only
+    // first ⌊T/C⌋ waves run whole tiles and the (tile, k-block) space of the last, partial
+    // wave is split evenly over the pairs (ranges of at least SK_MIN_SEG k-blocks); tile
+    // knob split=1 keeps whole tiles only
     const int CL = s->cl, NPP = CL / 2;
     // the persistent grid must be co-resident (stream-K finishers wait on other clusters):
     // at most the number of CL-CTA clusters the GPCs can hold at once (for CL = 4 fewer
@@ -1931,7 +2033,9 @@ mdh_status launch_t4(const Plan& p, const void* const* in, void* const* out, voi
     P.sk_pairs = 0;
     P.sk_w = 0;
     if (T % C != 0 && p.tiles.split != 1) {
-      const int nfull = R >= 1 ? (R - 1) * C : 0;
+      // every complete wave runs whole tiles (their epilogues overlap later MMAs); only the
+      // partial last wave is spread over all pairs, so few outputs are written at the end
+      const int nfull = R * C;
       const int64_t W = (int64_t)(T - nfull) * P.num_kb;
       const int sp = (int)std::min<int64_t>(std::min(C, t4::SK_MAX_PAIRS / NPP), W / t4::SK_MIN_SEG);
       if (sp >= 2) {
@@ -1939,7 +2043,7 @@ mdh_status launch_t4(const Plan& p, const void* const* in, void* const* out, voi
         P.sk_pairs = sp;
         P.sk_w = W;
         P.skpart = (float*)((char*)ws + s->tail_off);
-        P.skflag = (unsigned*)((char*)ws + s->tail_off + (size_t)t4::SK_MAX_PAIRS * 65536 * sizeof(float));
+        P.skflag = (unsigned*)((char*)ws + s->tail_off + (size_t)t4::SK_MAX_PAIRS * (s->nw / 256) * 65536 * sizeof(float));
       }
     }
     const int clusters = P.sk_pairs > 0 ? C : std::max(1, std::min(T, C));
@@ -1947,7 +2051,8 @@ mdh_status launch_t4(const Plan& p, const void* const* in, void* const* out, voi
     P.trace_n = P.trace ? clusters * NPP * (T / clusters + 4) : 0;
     const int grid2 = CL * clusters;
     P.c_vec4 = P.c_rowmajor && P.ldc % 4 == 0 && P.cbase % 4 == 0 && (uintptr_t)P.C % 16 == 0;
-    if (CL == 4) t4::gemm2_kernel<true, 4><<<grid2, t4::THREADS, t4::SMEM2_BYTES, st>>>(ma, mb, P);
+    if (s->nw == 512) t4::gemm2_kernel<true, 2, 512><<<grid2, t4::THREADS, t4::SMEM2_BYTES, st>>>(ma, mb, P);
+    else if (CL == 4) t4::gemm2_kernel<true, 4><<<grid2, t4::THREADS, t4::SMEM2_BYTES, st>>>(ma, mb, P);
     else t4::gemm2_kernel<true, 2><<<grid2, t4::THREADS, t4::SMEM2_BYTES, st>>>(ma, mb, P);
     return post_launch("t4_gemm2_kernel");
   }

@@ -161,7 +161,7 @@ void lookup_tiles(Plan* p, const char* table_path, const char* force) {
   Tiles t;
   // template defaults
   if (p->tmpl == T1_STENCIL) t.zchunk = 32;
-  if (p->tmpl == T4_TC) { t.bm = 128; t.bn = 256; t.bk = 64; t.stages = 4; t.cluster = 0; }   // cluster 0 = auto
+  if (p->tmpl == T4_TC) { t.bm = 128; t.bn = 0; t.bk = 64; t.stages = 4; t.cluster = 0; }   // bn, cluster 0 = auto
   std::string text;
   const char* path = table_path ? table_path : std::getenv("MDH_TILE_TABLE");
   if (path && *path) text = read_file(path);

@@ -470,14 +470,18 @@ def test_t4_split_tail_1sm(shape, tile, out):
                                              ((4096, 4096, 4096), None, "points"),   # 2 data-parallel waves + SK
                                              ((1024, 768, 640), "split=1", "full"),   # whole tiles only
                                              ((700, 1000, 1000), "cluster=4", "full"),  # odd row tiles: an idle pair
-                                             ((2500, 2000, 1000), "cluster=4", "points")])  # 4-CTA clusters
+                                             ((2500, 2000, 1000), "cluster=4", "points"),  # 4-CTA clusters
+                                             ((512, 768, 4096), "bn=512", "full"),    # wide 256x512 pair tiles
+                                             ((2500, 2000, 1000), "bn=512", "points"),
+                                             ((4096, 4096, 4096), "bn=512", "points")])
 def test_t4_stream_k(shape, tile, kind):
     """2-SM stream-K hybrid: whole-tile waves, then each cluster's even share of the remaining
     (tile, k-block) space; producers publish coalesced fp32 partials, the finisher (the one
     holding k = 0) adds them in k order.  Single pairs (default) and 4-CTA clusters
     (cluster=4: two pairs sharing B by TMA multicast; with an odd number of 256-row tiles
-    the last pair computes zero-filled rows and stores nothing).  Run twice on one plan:
-    the flags return to rest."""
+    the last pair computes zero-filled rows and stores nothing), and wide 256×512 pair
+    tiles (bn=512: two N=256 MMAs per k-step, per-column-half accumulator release).  Run
+    twice on one plan: the flags return to rest."""
     M, N, K = shape
     spec = S.matmul(M, N, K, "bf16")
     x = G.matmul_inputs(M, N, K, "bf16", "positive")
@@ -563,7 +567,9 @@ def test_fig3_paper_sizes(case):
 @pytest.mark.parametrize("cfg,tile", [((256, 7, 7, 512, 3, 3, 512), None),           # conv5_1, 2-SM
                                       ((3, 3, 5, 128, 3, 3, 64), None),              # P != Q, ragged M
                                       ((2, 9, 4, 256, 3, 3, 128), "cluster=1"),      # 1-SM kernel
-                                      ((64, 7, 7, 512, 3, 3, 512), "split=3"),       # 2-SM split-K tail
+                                      ((64, 7, 7, 512, 3, 3, 512), "bn=256"),        # narrow pair tiles, stream-K
+                                      ((64, 7, 7, 512, 3, 3, 512), "split=1"),       # wide pair tiles, whole tiles
+                                      ((3, 3, 5, 384, 3, 3, 64), "bn=512"),          # wide, ragged N
                                       ((5, 6, 6, 64, 2, 2, 64), None)])              # 2x2 window
 def test_mcc_im2col_tma(cfg, tile):
     """T4 A operand through a TMA im2col map (window origin walk with traversal strides,

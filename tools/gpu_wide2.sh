@@ -1,0 +1,16 @@
+cd $GRAFT_REPO_ROOT
+mkdir -p gpurun_out
+o=gpurun_out/wide2.txt
+: > $o
+MDH_DEBUG_SYNC=1 timeout 400 python -m pytest tests/test_gpu_parity.py -q -m gpu -x --timeout=120 -k "stream_k or im2col" >> $o 2>&1; echo "tests rc=$?" >> $o
+for ft in "bn=256" "bn=512" "split=1"; do
+echo "== $ft" >> $o
+timeout 200 python tools/time_one.py matmul_bf16 mcc_bf16 mm:12544,512,4608 mm:8192,8192,8192 --reps 20 --force-tile $ft 2>&1 | python -c "
+import sys, json
+for l in sys.stdin:
+    try: d = json.loads(l); print(d['workload'], d['ms'], d['value'], d['frac'])
+    except Exception: print(l.strip()[:200])" >> $o
+done
+timeout 200 python tools/t4_trace.py mm:4096,4096,4096 mm:12544,512,4608 mcc_bf16 > gpurun_out/trace_w2.jsonl 2>&1
+grep span gpurun_out/trace_w2.jsonl | cut -c1-260 >> $o
+tail -22 $o

@@ -48,10 +48,12 @@ def main():
         t0 = min(r[2] for r in tr)
         t_end = max(max(r[3], r[4]) for r in tr)
         units = []
-        for u, (sm, pair, a0, a1, e, wf, wa) in enumerate(tr):
+        for u, (sm, pair, a0, a1, e, wf, wa, ts, tp) in enumerate(tr):
             units.append({"u": u, "pair": pair, "sm": sm, "start_us": round((a0 - t0) / 1e3, 2),
                           "mma_us": round((a1 - a0) / 1e3, 2), "epi_done_us": round((e - t0) / 1e3, 2),
-                          "wait_full_kcyc": round(wf / 1e3, 1), "wait_acc_kcyc": round(wa / 1e3, 1)})
+                          "wait_full_kcyc": round(wf / 1e3, 1), "wait_acc_kcyc": round(wa / 1e3, 1),
+                          "seen_us": round((ts - t0) / 1e3, 2) if ts else None,
+                          "published_us": round((tp - t0) / 1e3, 2) if tp else None})
         pairs = {}
         for x in units:
             pairs.setdefault(x["pair"], []).append(x)
