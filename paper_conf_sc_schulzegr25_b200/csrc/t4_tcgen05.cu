@@ -837,14 +837,15 @@ struct SkIter {
   }
 };
 
-constexpr int S2 = 6;                          // stages (32 KB each)
+constexpr int S2 = 5;                          // stages (32 KB each)
 constexpr int A2_BYTES = 128 * BK * 2;         // this CTA's half of A (16 KB)
 constexpr int B2_BYTES = 128 * BK * 2;         // this CTA's half of B (16 KB)
 constexpr int STAGE2_BYTES = A2_BYTES + B2_BYTES;
-constexpr int STG2_BYTES = 8 * 32 * 32 * 4;    // epilogue staging: 32×32 fp32 per epilogue warp
-constexpr int S2W = 4;                         // stages of the wide (NW = 512) ring (48 KB each)
-constexpr int SMEM2_BYTES = S2 * STAGE2_BYTES + 1024 + 256 + STG2_BYTES;
+constexpr int STG2_BYTES = 2 * 8 * 32 * 32 * 4;  // epilogue staging: 2 × 32×32 fp32 per epilogue warp
+constexpr int S2W = 3;                         // stages of the wide (NW = 512) ring (48 KB each)
+constexpr int SMEM2_BYTES = S2 * STAGE2_BYTES + 1024 + 1024 + STG2_BYTES;   // ring, align slack, barriers, staging
 static_assert(S2W * (A2_BYTES + 2 * B2_BYTES) <= S2 * STAGE2_BYTES, "wide ring must fit the 2-SM smem budget");
+static_assert(SMEM2_BYTES <= 232448, "2-SM kernel exceeds 227 KB of shared memory");
 
 __device__ __forceinline__ uint32_t cluster_rank() {
   uint32_t r;
@@ -898,6 +899,12 @@ __device__ __forceinline__ void tma_load_2d_cg2_mc(uint32_t dst, const CUtensorM
       "l"((uint64_t)map), "r"(bar_cluster), "r"(c0), "r"(c1), "h"(mask)
       : "memory");
 }
+// TMA tensor store of a 32×32 fp32 box (128B-swizzled smem image) at {n, m}; OOB clipped
+__device__ __forceinline__ void tma_store_2d(const CUtensorMap* map, uint32_t src, int c0, int c1) {
+  asm volatile("cp.async.bulk.tensor.2d.global.shared::cta.bulk_group [%0, {%2, %3}], [%1];" ::"l"((uint64_t)map), "r"(src),
+               "r"(c0), "r"(c1)
+               : "memory");
+}
 __device__ __forceinline__ void mma_commit_cg2(uint32_t bar) {
   asm volatile(
       "{\n\t.reg .b16 m;\n\tmov.b16 m, 3;\n\t"
@@ -922,7 +929,7 @@ __device__ __forceinline__ void mbar_arrive_cluster(uint32_t bar_cluster) {
 template <bool OUT_ROWMAJOR, int CL, int NW = 256>
 __global__ void __cluster_dims__(CL, 1, 1) __launch_bounds__(THREADS, 1)
     gemm2_kernel(const __grid_constant__ CUtensorMap mapA, const __grid_constant__ CUtensorMap mapB,
-                 const __grid_constant__ Params P) {
+                 const __grid_constant__ CUtensorMap mapC, const __grid_constant__ Params P) {
   extern __shared__ __align__(1024) uint8_t smem_raw[];
   constexpr int NH = NW / 256;                   // N=256 MMAs per k-step
   constexpr int NS = NW == 512 ? S2W : S2;       // ring stages
@@ -947,6 +954,7 @@ __global__ void __cluster_dims__(CL, 1, 1) __launch_bounds__(THREADS, 1)
   if (warp == 0 && lane == 0) {
     asm volatile("prefetch.tensormap [%0];" ::"l"((uint64_t)&mapA) : "memory");
     asm volatile("prefetch.tensormap [%0];" ::"l"((uint64_t)&mapB) : "memory");
+    if (P.c_vec4) asm volatile("prefetch.tensormap [%0];" ::"l"((uint64_t)&mapC) : "memory");
     for (int s = 0; s < NS; ++s) {
       mbar_init(full0 + 8 * s, 2);
       mbar_init(empty0 + 8 * s, NPP);
@@ -1094,7 +1102,9 @@ __global__ void __cluster_dims__(CL, 1, 1) __launch_bounds__(THREADS, 1)
     const int half = (warp - 2) >> 2;
     const int row = quad * 32 + lane;
     const int ew = rank * 8 + (warp - 2);          // this warp's slot in a stream-K partial
-    const uint32_t stg = smem_u32(smem + NS * (A2_BYTES + BSTG) + 256) + (warp - 2) * 4096;
+    // (1024-byte aligned: the TMA 128B swizzle pattern is a function of the address bits)
+    const uint32_t stg0 = smem_u32(smem + NS * (A2_BYTES + BSTG) + 1024) + (warp - 2) * 8192;
+    int sbuf = 0;                                  // staging buffer of the next TMA store
     const uint32_t tempty_leader = map_to_rank(tempty0, 2 * pp);
     int it = 0;
     SkIter wi(P, cluster_id, nclusters);
@@ -1159,37 +1169,25 @@ __global__ void __cluster_dims__(CL, 1, 1) __launch_bounds__(THREADS, 1)
           }
         }
         if (OUT_ROWMAJOR && P.c_vec4) {
-          // transpose through this warp's swizzled 32×32 staging tile (16-byte chunk j of row
-          // r at (j ^ (r & 7))·16: conflict-free both ways), then 8 stores in which 8 lanes
-          // cover one 128-byte row segment, i.e. 4 whole lines per instruction
+          // this warp's 32 rows × 32 columns into a 128B-swizzled staging image (16-byte chunk
+          // j of row r at (j ^ (r & 7))·16: conflict-free), then one TMA tensor store of the
+          // 32×32 box (rows / columns beyond M / N are clipped by the TMA unit); two staging
+          // buffers per warp, so a buffer is rewritten only after its previous store read it
+          const uint32_t stg = stg0 + sbuf * 4096;
+          if (lane == 0) asm volatile("cp.async.bulk.wait_group.read 1;" ::: "memory");
+          __syncwarp();
 #pragma unroll
           for (int j = 0; j < 8; ++j)
             asm volatile("st.shared.v4.b32 [%0], {%1, %2, %3, %4};" ::"r"(stg + lane * 128 + ((j ^ (lane & 7)) << 4)),
                          "r"(r[4 * j]), "r"(r[4 * j + 1]), "r"(r[4 * j + 2]), "r"(r[4 * j + 3])
                          : "memory");
+          fence_proxy_async();
           __syncwarp();
-          const int cj = lane & 7;
-          const int64_t ncol = nb + 4 * cj;
-#pragma unroll
-          for (int i = 0; i < 8; ++i) {
-            const int rr = 4 * i + (lane >> 3);
-            const int64_t mm = m - row + quad * 32 + rr;     // this CTA's row quad*32 + rr
-            float4 v;
-            asm volatile("ld.shared.v4.f32 {%0, %1, %2, %3}, [%4];"
-                         : "=f"(v.x), "=f"(v.y), "=f"(v.z), "=f"(v.w)
-                         : "r"(stg + rr * 128 + ((cj ^ (rr & 7)) << 4)));
-            if (mm < P.M) {
-              float* dst = P.C + P.cbase + mm * P.ldc + ncol;
-              if (ncol + 4 <= P.N) {
-                *reinterpret_cast<float4*>(dst) = v;
-              } else {
-                if (ncol < P.N) dst[0] = v.x;
-                if (ncol + 1 < P.N) dst[1] = v.y;
-                if (ncol + 2 < P.N) dst[2] = v.z;
-              }
-            }
+          if (lane == 0) {
+            tma_store_2d(&mapC, stg, (int)nb, (int)(m - row + quad * 32));
+            asm volatile("cp.async.bulk.commit_group;" ::: "memory");
           }
-          __syncwarp();
+          sbuf ^= 1;
         } else if (OUT_ROWMAJOR && mok && nb + 32 <= P.N && ((crow + nb) & 3) == 0) {
           float4* dst = reinterpret_cast<float4*>(P.C + crow + nb);
 #pragma unroll
@@ -1247,6 +1245,7 @@ __global__ void __cluster_dims__(CL, 1, 1) __launch_bounds__(THREADS, 1)
       if (P.trace && leader && warp == 2 && lane == 0 && pair_gid + it * nclusters * NPP < P.trace_n)
         P.trace[8 * (pair_gid + it * nclusters * NPP) + 3] = gtimer();
     }
+    if (lane == 0) asm volatile("cp.async.bulk.wait_group 0;" ::: "memory");   // stores done before exit
   }
   __syncwarp();                  // lanes 1..31 of warps 0/1 wait for their role lane
   tc_fence_before();
@@ -2050,10 +2049,25 @@ mdh_status launch_t4(const Plan& p, const void* const* in, void* const* out, voi
     P.trace = t4_trace_buffer(clusters * NPP * (T / clusters + 4));
     P.trace_n = P.trace ? clusters * NPP * (T / clusters + 4) : 0;
     const int grid2 = CL * clusters;
-    P.c_vec4 = P.c_rowmajor && P.ldc % 4 == 0 && P.cbase % 4 == 0 && (uintptr_t)P.C % 16 == 0;
-    if (s->nw == 512) t4::gemm2_kernel<true, 2, 512><<<grid2, t4::THREADS, t4::SMEM2_BYTES, st>>>(ma, mb, P);
-    else if (CL == 4) t4::gemm2_kernel<true, 4><<<grid2, t4::THREADS, t4::SMEM2_BYTES, st>>>(ma, mb, P);
-    else t4::gemm2_kernel<true, 2><<<grid2, t4::THREADS, t4::SMEM2_BYTES, st>>>(ma, mb, P);
+    P.c_vec4 = P.c_rowmajor && P.ldc % 4 == 0 && P.cbase % 4 == 0 && (uintptr_t)P.C % 16 == 0 && P.M < INT32_MAX &&
+               P.N < INT32_MAX;
+    CUtensorMap mc;
+    memset(&mc, 0, sizeof(mc));
+    if (P.c_vec4) {
+      auto fn = encode_fn();
+      if (!fn) { set_error("cuTensorMapEncodeTiled unavailable (driver too old?)"); return MDH_ERR_CUDA; }
+      cuuint64_t dims[2] = {(cuuint64_t)P.N, (cuuint64_t)P.M};
+      cuuint64_t strides[1] = {(cuuint64_t)P.ldc * 4};
+      cuuint32_t box[2] = {32, 32};
+      cuuint32_t estr[2] = {1, 1};
+      CUresult r = fn(&mc, CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 2, (void*)(P.C + P.cbase), dims, strides, box, estr,
+                      CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_128B, CU_TENSOR_MAP_L2_PROMOTION_NONE,
+                      CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+      if (r != CUDA_SUCCESS) { set_error("cuTensorMapEncodeTiled (C store map) failed (%d)", (int)r); return MDH_ERR_CUDA; }
+    }
+    if (s->nw == 512) t4::gemm2_kernel<true, 2, 512><<<grid2, t4::THREADS, t4::SMEM2_BYTES, st>>>(ma, mb, mc, P);
+    else if (CL == 4) t4::gemm2_kernel<true, 4><<<grid2, t4::THREADS, t4::SMEM2_BYTES, st>>>(ma, mb, mc, P);
+    else t4::gemm2_kernel<true, 2><<<grid2, t4::THREADS, t4::SMEM2_BYTES, st>>>(ma, mb, mc, P);
     return post_launch("t4_gemm2_kernel");
   }
   int grid = std::min(P.num_tiles, sms);
