@@ -222,9 +222,11 @@ int32_t mdh_last_launch_count(void);
  * host[8u..8u+7]: (SM id << 32 | CTA-pair id, %globaltimer ns at the unit's first MMA
  * issue, at its last MMA commit, at the end of its epilogue, SM cycles the MMA issuer
  * waited for loaded stages, SM cycles it waited for a free accumulator, %globaltimer when a
- * stream-K finisher saw all its partials, when a producer published its partial; else 0).  Synchronises the device,
- * copies at most max_units units and returns how many; 0 when tracing is off, -1 on a
- * CUDA error.  `host` is caller-owned.                                                  */
+ * stream-K finisher saw all its partials, when a producer published its partial; else 0).  When
+ * all n traced units fit (n ≤ max_units), 1024 more u64 follow at host[8n..]: per CTA pair
+ * p < 256 and CTA r of the pair, %globaltimer at kernel entry [2p + 512r] and exit
+ * [2p + 1 + 512r]; `host` must then hold 8·max_units + 1024 u64.  Synchronises the device,
+ * returns n; 0 when tracing is off, -1 on a CUDA error.  `host` is caller-owned.         */
 int64_t mdh_debug_t4_trace(uint64_t* host, int64_t max_units);
 
 #ifdef __cplusplus

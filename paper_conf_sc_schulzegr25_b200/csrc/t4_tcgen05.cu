@@ -950,6 +950,7 @@ __global__ void __cluster_dims__(CL, 1, 1) __launch_bounds__(THREADS, 1)
   // pair tiles: tiles_m/tiles_n count 256×NW tiles; clusters stride over them
   const int cluster_id = blockIdx.x / CL, nclusters = gridDim.x / CL;
   const int pair_gid = cluster_id * NPP + (int)pp;   // partial slot / trace row of this pair
+  if (P.trace && threadIdx.x == 0 && pair_gid < 256) P.trace[8 * P.trace_n + 2 * pair_gid + rank * 512] = gtimer();
 
   if (warp == 0 && lane == 0) {
     asm volatile("prefetch.tensormap [%0];" ::"l"((uint64_t)&mapA) : "memory");
@@ -1254,6 +1255,7 @@ __global__ void __cluster_dims__(CL, 1, 1) __launch_bounds__(THREADS, 1)
     tc_fence_after();
     asm volatile("tcgen05.dealloc.cta_group::2.sync.aligned.b32 %0, %1;" ::"r"(tmem), "r"(TMEM_COLS));
   }
+  if (P.trace && threadIdx.x == 0 && pair_gid < 256) P.trace[8 * P.trace_n + 2 * pair_gid + 1 + rank * 512] = gtimer();
 }
 
 constexpr int SK_MAX_PAIRS = 74;     // stream-K partial slots reserved in the workspace (2-SM path)
@@ -1849,12 +1851,13 @@ static mdh_status make_im2col_map(CUtensorMap* map, const void* base, const T4St
 // 2-SM launch, read back by mdh_debug_t4_trace
 static unsigned long long* g_trace = nullptr;
 static int g_trace_units = 0;
+static int g_trace_used = 0;     // trace_n of the last traced launch (its entry/exit block follows)
 static unsigned long long* t4_trace_buffer(int units) {
   static const bool on = std::getenv("MDH_T4_TRACE") && std::getenv("MDH_T4_TRACE")[0] == '1';
   if (!on) return nullptr;
   if (units > g_trace_units) {
     if (g_trace) cudaFree(g_trace);
-    if (cudaMalloc(&g_trace, (size_t)units * 8 * sizeof(unsigned long long)) != cudaSuccess) {
+    if (cudaMalloc(&g_trace, ((size_t)units * 8 + 1024) * sizeof(unsigned long long)) != cudaSuccess) {
       cudaGetLastError();
       g_trace = nullptr;
       g_trace_units = 0;
@@ -1862,7 +1865,8 @@ static unsigned long long* t4_trace_buffer(int units) {
     }
     g_trace_units = units;
   }
-  cudaMemset(g_trace, 0, (size_t)g_trace_units * 8 * sizeof(unsigned long long));
+  cudaMemset(g_trace, 0, ((size_t)g_trace_units * 8 + 1024) * sizeof(unsigned long long));
+  g_trace_used = units;
   return g_trace;
 }
 
@@ -2046,8 +2050,9 @@ mdh_status launch_t4(const Plan& p, const void* const* in, void* const* out, voi
       }
     }
     const int clusters = P.sk_pairs > 0 ? C : std::max(1, std::min(T, C));
-    P.trace = t4_trace_buffer(clusters * NPP * (T / clusters + 4));
-    P.trace_n = P.trace ? clusters * NPP * (T / clusters + 4) : 0;
+    P.trace_n = clusters * NPP * (T / clusters + 4);
+    P.trace = t4_trace_buffer(P.trace_n);
+    if (!P.trace) P.trace_n = 0;
     const int grid2 = CL * clusters;
     P.c_vec4 = P.c_rowmajor && P.ldc % 4 == 0 && P.cbase % 4 == 0 && (uintptr_t)P.C % 16 == 0 && P.M < INT32_MAX &&
                P.N < INT32_MAX;
@@ -2108,9 +2113,14 @@ mdh_status launch_t4(const Plan& p, const void* const* in, void* const* out, voi
 
 extern "C" int64_t mdh_debug_t4_trace(uint64_t* host, int64_t max_units) {
   if (!mdh::g_trace || !host) return 0;
-  const int64_t n = std::min<int64_t>(max_units, mdh::g_trace_units);
+  const int64_t n = std::min<int64_t>(max_units, mdh::g_trace_used);
   if (cudaDeviceSynchronize() != cudaSuccess ||
       cudaMemcpy(host, mdh::g_trace, (size_t)n * 8 * sizeof(uint64_t), cudaMemcpyDeviceToHost) != cudaSuccess) {
+    cudaGetLastError();
+    return -1;
+  }
+  if (n == mdh::g_trace_used &&
+      cudaMemcpy(host + 8 * n, mdh::g_trace + 8 * n, 1024 * sizeof(uint64_t), cudaMemcpyDeviceToHost) != cudaSuccess) {
     cudaGetLastError();
     return -1;
   }

@@ -289,13 +289,15 @@ class Plan:
         """Diagnostics: the T4 2-SM per-unit timeline of the last launch (MDH_T4_TRACE=1),
         as a list of (sm, pair, t_first_mma, t_last_commit, t_epilogue_done) in ns and
         (wait_full, wait_accumulator) in SM cycles, then (t_partials_seen, t_partial_published)
-        in ns (stream-K finisher / producer units, else 0)."""
-        buf = (ctypes.c_uint64 * (8 * max_units))()
+        in ns (stream-K finisher / producer units, else 0); and per CTA its (entry, exit) times."""
+        buf = (ctypes.c_uint64 * (8 * max_units + 1024))()
         n = int(lib().mdh_debug_t4_trace(buf, max_units))
         if n < 0:
             raise MdhError(-1, "mdh_debug_t4_trace failed")
-        return [(buf[8 * u] >> 32, buf[8 * u] & 0xffffffff, buf[8 * u + 1], buf[8 * u + 2], buf[8 * u + 3],
-                 buf[8 * u + 4], buf[8 * u + 5], buf[8 * u + 6], buf[8 * u + 7]) for u in range(n) if buf[8 * u + 1]]
+        units = [(buf[8 * u] >> 32, buf[8 * u] & 0xffffffff, buf[8 * u + 1], buf[8 * u + 2], buf[8 * u + 3],
+                  buf[8 * u + 4], buf[8 * u + 5], buf[8 * u + 6], buf[8 * u + 7]) for u in range(n) if buf[8 * u + 1]]
+        ee = [(buf[8 * n + i], buf[8 * n + i + 1]) for r in (0, 512) for i in range(r, r + 512, 2) if buf[8 * n + i]]
+        return units, ee
 
 
 class Comm:

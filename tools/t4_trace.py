@@ -41,7 +41,7 @@ def main():
             torch.cuda.synchronize()
             plan(tin, outs)
             torch.cuda.synchronize()
-        tr = Plan.t4_trace()
+        tr, ee = Plan.t4_trace()
         if not tr:
             print(json.dumps({"workload": name, "trace": "empty (not the 2-SM kernel?)"}))
             continue
@@ -59,7 +59,13 @@ def main():
             pairs.setdefault(x["pair"], []).append(x)
         busy = sorted(round(sum(y["mma_us"] for y in v), 1) for v in pairs.values())
         ends = sorted(max(y["epi_done_us"] for y in v) for v in pairs.values())
-        print(json.dumps({"workload": name, "span_us": round((t_end - t0) / 1e3, 2), "units": len(units),
+        k0 = min(e[0] for e in ee) if ee else t0
+        k1 = max(e[1] for e in ee) if ee else t_end
+        print(json.dumps({"workload": name, "kernel_us": round((k1 - k0) / 1e3, 2),
+                          "entry_spread_us": round((max(e[0] for e in ee) - k0) / 1e3, 2) if ee else None,
+                          "first_mma_after_entry_us": round((t0 - k0) / 1e3, 2),
+                          "exit_after_last_epilogue_us": round((k1 - t_end) / 1e3, 2),
+                          "span_us": round((t_end - t0) / 1e3, 2), "units": len(units),
                           "pairs": len(pairs), "pair_busy_us_min_med_max": [busy[0], busy[len(busy) // 2], busy[-1]],
                           "pair_end_us_min_med_max": [ends[0], ends[len(ends) // 2], ends[-1]],
                           "wait_full_kcyc_total": round(sum(x["wait_full_kcyc"] for x in units), 1),
