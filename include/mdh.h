@@ -37,7 +37,7 @@
 extern "C" {
 #endif
 
-#define MDH_ABI_VERSION 2  /* 2: MDH_MAX_ACC 8 -> 32 */
+#define MDH_ABI_VERSION 3  /* 2: MDH_MAX_ACC 8 -> 32; 3: mdh_stencil_sweeps */
 
 #define MDH_MAX_D     10  /* MCC_Caps is 10-D (Fig 3); configs need <= 7        */
 #define MDH_MAX_RANK   8  /* buffer rank                                                */
@@ -202,6 +202,41 @@ mdh_status mdh_combine_partials(mdh_plan_t plan, const void* const* partial_outs
                                 int32_t S, void* const* out, void* cuda_stream);
 
 mdh_status mdh_destroy(mdh_plan_t plan);
+
+/* ---- Stencil time-stepping with a halo exchange (reading C-34).
+ * The paper evaluates one Jacobi sweep; time-stepping applies the same md_hom
+ * repeatedly: sweep t reads buffer src_t and writes dst_t (u→v, v→u, …).
+ *
+ * `plan` must be an all-cc map with one input and one output buffer of the same dtype and
+ * the same shape [nz, …] (e.g. mdh_workloads.specs.jacobi3d_sweep, whose output index
+ * function is the input's centre access): its output image is the interior, the rest of
+ * the output buffer (the boundary shell) is never written (C-5), so u and v must both
+ * hold the fixed boundary on entry.  Buffer dim 0 is the sharded dim: plane = the
+ * product of the other extents; the stencil may reach at most one plane below / above
+ * (halo width 1).  With halo == NULL or world == 1 this is the whole domain.  Otherwise
+ * this rank owns local planes 1..nz-2 of a z-slab, plane 0 / nz-1 being halo copies of
+ * the lower / upper neighbour's last / first owned plane; after every sweep the first and
+ * last owned planes of dst go to the neighbours' halo planes of their dst:
+ *   - NCCL transport (nccl_comm from mdh_comm_init; one process per GPU): grouped
+ *     ncclSend/ncclRecv on `cuda_stream`, any number of sweeps per call;
+ *   - peer transport (nccl_comm NULL): device-to-device copies into peer_lo / peer_hi,
+ *     the neighbours' halo planes (addresses this process can write: same device, P2P or
+ *     CUDA-IPC mapped).  The caller orders the ranks' calls (one sweep per call, lock-step —
+ *     e.g. virtual ranks on one stream).
+ * `workspace` as for mdh_execute.  On return *result_in_v = sweeps odd (the final field
+ * is in v), else 0 (in u).  Errors: MDH_ERR_INVALID_ARG (bad plan shape, aliasing u/v,
+ * sweeps < 0, missing transport, nz < 3), MDH_ERR_NCCL, MDH_ERR_CUDA.                  */
+typedef struct mdh_halo {
+  void* nccl_comm;    /* NCCL transport, or NULL                                        */
+  int32_t rank;       /* this slab's index along dim 0 (neighbours rank-1, rank+1)      */
+  int32_t world;      /* number of slabs                                                */
+  void* peer_lo[2];   /* peer transport: lower neighbour's TOP halo plane in its u [0] and v [1] (NULL at rank 0)   */
+  void* peer_hi[2];   /* peer transport: upper neighbour's BOTTOM halo plane in its u and v (NULL at rank world-1) */
+} mdh_halo;
+
+mdh_status mdh_stencil_sweeps(mdh_plan_t plan, void* u, void* v, int32_t sweeps, const mdh_halo* halo,
+                              void* workspace, size_t workspace_bytes, void* cuda_stream,
+                              int32_t* result_in_v);
 
 /* NCCL communicator bootstrap (NCCL is loaded with dlopen on first use).
  * id128: 128 bytes (ncclUniqueId) produced on one rank and broadcast by the caller. */

@@ -10,4 +10,4 @@ the mathematics; parity with the AUTHORS' code is unpinned for the readings C-16
 C-18, C-19, C-21, C-22 because the paper prints no computed values.
 """
 from .oracle import (evaluate, evaluate_points, shapes, combine_tuple, build,  # noqa: F401
-                     max_threads, random_points, OracleError)
+                     max_threads, random_points, stencil_sweeps, OracleError)

@@ -184,3 +184,20 @@ def random_points(spec: dict, n: int, seed: int = 7) -> np.ndarray:
         if o == "CC":
             pts[:, d] = g.integers(0, s, size=n)
     return pts
+
+
+def stencil_sweeps(spec: dict, u0: np.ndarray, sweeps: int, threads: int = 0) -> np.ndarray:
+    """`sweeps` applications of a same-shape all-cc map (reading C-34):
+    u_{t+1} = md_hom(f, cc…)(u_t) on the image of the output index function, u_t elsewhere
+    (the fixed boundary, reading C-5).  A plain loop over evaluate(); the state is kept in
+    fp64 (the spec is re-typed to f64 after the first application).  Returns fp64."""
+    if len(spec["inputs"]) != 1 or len(spec["outputs"]) != 1 or any(o != "CC" for o in spec["ops"]):
+        raise OracleError("stencil_sweeps needs one input, one output and only cc dims")
+    sp64 = {**spec, "inputs": [{**spec["inputs"][0], "dtype": "f64"}],
+            "outputs": [{**spec["outputs"][0], "dtype": "f64"}]}
+    u = np.ascontiguousarray(u0, np.float64).copy()
+    for _ in range(sweeps):
+        nxt = evaluate(sp64, [u], threads=threads, fill=np.nan)[0].reshape(u.shape)
+        u = np.where(np.isnan(nxt), u, nxt)
+    return u
+

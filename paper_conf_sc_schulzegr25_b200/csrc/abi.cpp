@@ -296,6 +296,62 @@ mdh_status mdh_combine_partials(mdh_plan_t plan, const void* const* partial_outs
   return mdh::launch_combine(p, partial_outs, S, out, (cudaStream_t)cuda_stream);
 }
 
+mdh_status mdh_stencil_sweeps(mdh_plan_t plan, void* u, void* v, int32_t sweeps, const mdh_halo* halo,
+                              void* workspace, size_t workspace_bytes, void* cuda_stream, int32_t* result_in_v) {
+  mdh::reset_launch_count();
+  if (!plan || !u || !v || sweeps < 0) { set_error("bad arguments (plan, u, v, sweeps >= 0)"); return MDH_ERR_INVALID_ARG; }
+  const mdh::Plan& p = plan->p;
+  if (p.n_in != 1 || p.n_out != 1 || p.nred != 0 || p.nps != 0) {
+    set_error("stencil sweeps need an all-cc plan with one input and one output buffer");
+    return MDH_ERR_INVALID_ARG;
+  }
+  const mdh::Buf& I = p.in[0];
+  const mdh::Buf& O = p.out[0];
+  bool same = I.dtype == O.dtype && I.rank == O.rank && I.elems == O.elems;
+  for (int r = 0; same && r < I.rank; ++r) same = I.shape[r] == O.shape[r];
+  if (!same || I.rank < 2) {
+    set_error("stencil sweeps: input and output buffers must have the same dtype and shape (rank >= 2)");
+    return MDH_ERR_INVALID_ARG;
+  }
+  const int64_t nz = I.shape[0];
+  const size_t plane = (size_t)(I.elems / nz) * mdh::dtype_size(I.dtype);
+  const int world = halo ? halo->world : 1, rank = halo ? halo->rank : 0;
+  if (world < 1 || rank < 0 || rank >= world) { set_error("bad halo rank/world"); return MDH_ERR_INVALID_ARG; }
+  const bool nccl = world > 1 && halo->nccl_comm;
+  if (world > 1 && nz < 3) { set_error("a slab needs >= 3 planes (halo, owned, halo)"); return MDH_ERR_INVALID_ARG; }
+  if (world > 1 && !nccl) {
+    if ((rank > 0 && (!halo->peer_lo[0] || !halo->peer_lo[1])) ||
+        (rank < world - 1 && (!halo->peer_hi[0] || !halo->peer_hi[1]))) {
+      set_error("stencil sweeps: world > 1 needs nccl_comm or the neighbours' halo-plane addresses");
+      return MDH_ERR_INVALID_ARG;
+    }
+  }
+  cudaStream_t st = (cudaStream_t)cuda_stream;
+  char* buf[2] = {(char*)u, (char*)v};
+  int launches = 0;
+  for (int t = 0; t < sweeps; ++t) {
+    const int s = t & 1, d = s ^ 1;
+    const void* in[1] = {buf[s]};
+    void* out[1] = {buf[d]};
+    mdh_status e = mdh_execute(plan, in, out, workspace, workspace_bytes, cuda_stream);
+    if (e != MDH_OK) return e;
+    launches += mdh::launch_count();
+    if (world > 1) {
+      if (nccl) {
+        MDH_TRY(mdh::comm_halo_exchange(halo->nccl_comm, rank, world, buf[d], plane, nz, st));
+      } else {
+        if (rank > 0) MDH_CUDA(cudaMemcpyAsync(halo->peer_lo[d], buf[d] + plane, plane, cudaMemcpyDeviceToDevice, st));
+        if (rank < world - 1)
+          MDH_CUDA(cudaMemcpyAsync(halo->peer_hi[d], buf[d] + (nz - 2) * plane, plane, cudaMemcpyDeviceToDevice, st));
+      }
+    }
+  }
+  mdh::reset_launch_count();
+  mdh::count_launch(launches);
+  if (result_in_v) *result_in_v = sweeps & 1;
+  return MDH_OK;
+}
+
 mdh_status mdh_destroy(mdh_plan_t plan) {
   if (!plan) return MDH_OK;
   if (plan->p.dconst) {

@@ -21,6 +21,10 @@ struct Nccl {
   ncclResult_t (*allGather)(const void*, void*, size_t, ncclDataType_t, ncclComm_t, cudaStream_t) = nullptr;
   ncclResult_t (*allReduce)(const void*, void*, size_t, ncclDataType_t, ncclRedOp_t, ncclComm_t, cudaStream_t) = nullptr;
   const char* (*getErrorString)(ncclResult_t) = nullptr;
+  ncclResult_t (*send)(const void*, size_t, ncclDataType_t, int, ncclComm_t, cudaStream_t) = nullptr;
+  ncclResult_t (*recv)(void*, size_t, ncclDataType_t, int, ncclComm_t, cudaStream_t) = nullptr;
+  ncclResult_t (*groupStart)() = nullptr;
+  ncclResult_t (*groupEnd)() = nullptr;
   bool ok = false;
 };
 Nccl g_nccl;
@@ -40,6 +44,10 @@ void load() {
   SYM(allGather, "ncclAllGather");
   SYM(allReduce, "ncclAllReduce");
   SYM(getErrorString, "ncclGetErrorString");
+  SYM(send, "ncclSend");
+  SYM(recv, "ncclRecv");
+  SYM(groupStart, "ncclGroupStart");
+  SYM(groupEnd, "ncclGroupEnd");
 #undef SYM
   g_nccl.ok = g_nccl.getUniqueId && g_nccl.commInitRank && g_nccl.commDestroy && g_nccl.allGather &&
               g_nccl.allReduce && g_nccl.getErrorString;
@@ -109,6 +117,30 @@ mdh_status comm_allreduce(void* comm, const void* send, void* recv, size_t count
   }
   ncclRedOp_t o = op == MDH_PW_ADD ? ncclSum : (op == MDH_PW_MAX ? ncclMax : ncclMin);
   return chk(g_nccl.allReduce(send, recv, count, t, o, (ncclComm_t)comm, st), "ncclAllReduce");
+}
+
+// Halo exchange of a z-slab after a sweep (reading C-34): my first owned plane
+// (local plane 1) to the lower neighbour, whose copy lands in my plane 0 from it, and my
+// last owned plane (nz-2) to the upper neighbour / plane nz-1 from it.  One NCCL group, so
+// the four point-to-point transfers proceed together over NVLink.
+mdh_status comm_halo_exchange(void* comm, int rank, int world, char* buf, size_t plane_bytes, int64_t nz,
+                              cudaStream_t st) {
+  MDH_TRY(need());
+  if (!g_nccl.send || !g_nccl.recv || !g_nccl.groupStart || !g_nccl.groupEnd) {
+    set_error("this NCCL has no ncclSend/ncclRecv (needs >= 2.7)");
+    return MDH_ERR_NCCL;
+  }
+  ncclComm_t c = (ncclComm_t)comm;
+  MDH_TRY(chk(g_nccl.groupStart(), "ncclGroupStart"));
+  if (rank > 0) {
+    MDH_TRY(chk(g_nccl.send(buf + plane_bytes, plane_bytes, ncclUint8, rank - 1, c, st), "ncclSend"));
+    MDH_TRY(chk(g_nccl.recv(buf, plane_bytes, ncclUint8, rank - 1, c, st), "ncclRecv"));
+  }
+  if (rank < world - 1) {
+    MDH_TRY(chk(g_nccl.send(buf + (nz - 2) * plane_bytes, plane_bytes, ncclUint8, rank + 1, c, st), "ncclSend"));
+    MDH_TRY(chk(g_nccl.recv(buf + (nz - 1) * plane_bytes, plane_bytes, ncclUint8, rank + 1, c, st), "ncclRecv"));
+  }
+  return chk(g_nccl.groupEnd(), "ncclGroupEnd");
 }
 
 }  // namespace mdh

@@ -176,6 +176,8 @@ mdh_status comm_unique_id(void* id128);
 mdh_status comm_init(const void* id128, int world, int rank, int device, void** comm);
 mdh_status comm_destroy(void* comm);
 mdh_status comm_allgather(void* comm, const void* send, void* recv, size_t bytes, cudaStream_t st);
+mdh_status comm_halo_exchange(void* comm, int rank, int world, char* buf, size_t plane_bytes, int64_t nz,
+                              cudaStream_t st);
 mdh_status comm_allreduce(void* comm, const void* send, void* recv, size_t count, mdh_dtype dt,
                           mdh_combine op, cudaStream_t st);
 

@@ -18,7 +18,7 @@ import threading
 import numpy as np
 
 MAX_D, MAX_RANK, MAX_ACC, MAX_BUFS = 10, 8, 32, 32
-ABI_VERSION = 2                    # include/mdh.h MDH_ABI_VERSION
+ABI_VERSION = 3                    # include/mdh.h MDH_ABI_VERSION
 HERE = os.path.dirname(os.path.abspath(__file__))
 LIB_PATH = os.path.join(HERE, "libmdh.so")
 
@@ -52,6 +52,12 @@ class PlanOpts(ctypes.Structure):
     _fields_ = [("device", ctypes.c_int32), ("world_size", ctypes.c_int32), ("rank", ctypes.c_int32),
                 ("nccl_comm", ctypes.c_void_p), ("shard_dim", ctypes.c_int32), ("flags", ctypes.c_uint32),
                 ("tile_table", ctypes.c_char_p), ("force_tile", ctypes.c_char_p)]
+
+
+class Halo(ctypes.Structure):
+    """mdh_halo (include/mdh.h): the z-slab neighbourhood of a stencil time-stepping rank."""
+    _fields_ = [("nccl_comm", ctypes.c_void_p), ("rank", ctypes.c_int32), ("world", ctypes.c_int32),
+                ("peer_lo", ctypes.c_void_p * 2), ("peer_hi", ctypes.c_void_p * 2)]
 
 
 class MdhError(RuntimeError):
@@ -93,12 +99,14 @@ def lib():
             L.mdh_last_error.restype = ctypes.c_char_p
             L.mdh_abi_version.restype = ctypes.c_int32
             L.mdh_last_launch_count.restype = ctypes.c_int32
+            L.mdh_stencil_sweeps.argtypes = [P, P, P, ctypes.c_int32, ctypes.POINTER(Halo), P, S, P,
+                                             ctypes.POINTER(ctypes.c_int32)]
             L.mdh_debug_t4_trace.argtypes = [P, ctypes.c_int64]
             L.mdh_debug_t4_trace.restype = ctypes.c_int64
             for name in ("mdh_plan", "mdh_plan_workspace_size", "mdh_plan_local_shape", "mdh_plan_describe",
                          "mdh_execute", "mdh_plan_host_scratch_size", "mdh_execute_host",
                          "mdh_combine_partials", "mdh_destroy", "mdh_comm_unique_id", "mdh_comm_init",
-                         "mdh_comm_destroy"):
+                         "mdh_comm_destroy", "mdh_stencil_sweeps"):
                 getattr(L, name).restype = ctypes.c_int
             if L.mdh_abi_version() != ABI_VERSION:
                 raise RuntimeError(f"{LIB_PATH}: ABI version {L.mdh_abi_version()} != {ABI_VERSION} (stale build?)")
@@ -279,6 +287,18 @@ class Plan:
         st = stream if stream is not None else torch.cuda.current_stream(outputs[0].device).cuda_stream
         _check(lib().mdh_combine_partials(self._h, pp, len(partials), op, st))
         return outputs
+
+    def stencil_sweeps(self, u, v, sweeps: int, halo: "Halo | None" = None, stream=None, workspace_ptr=None):
+        """Time-stepping (mdh_stencil_sweeps): `sweeps` applications u→v→u…, with the halo
+        exchange of `halo` after each; returns the tensor holding the final field."""
+        import torch
+        ws = workspace_ptr if workspace_ptr is not None else (self.workspace() if self.workspace_bytes else None)
+        st = stream if stream is not None else torch.cuda.current_stream(u.device).cuda_stream
+        res = ctypes.c_int32()
+        _check(lib().mdh_stencil_sweeps(self._h, u.data_ptr(), v.data_ptr(), sweeps,
+                                        ctypes.byref(halo) if halo is not None else None, ws, self.workspace_bytes,
+                                        st, ctypes.byref(res)))
+        return v if res.value else u
 
     @staticmethod
     def last_launch_count() -> int:

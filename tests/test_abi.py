@@ -32,7 +32,7 @@ def test_library_exports_every_header_symbol(mdh):
     L = ctypes.CDLL(mdh.library_path())
     for n in names:
         assert hasattr(L, n), n
-    assert mdh.abi_version() == 2
+    assert mdh.abi_version() == 3
 
 
 def plan_status(mdh, spec, **kw):

@@ -142,3 +142,73 @@ def test_sharded_plans_reassemble(name, world):
         msgs.append(q.get())
     assert all(pr.exitcode == 0 for pr in procs), msgs
     assert "ok" in msgs, msgs
+
+
+def _sweeps_worker(rank, world, port, q):
+    """One z-slab of a Jacobi_3D time-stepping run (reading C-34): the rank's slab with one
+    halo plane per side, swept by the oracle, and after every sweep the exchange
+    mdh_stencil_sweeps performs — first owned plane (1) to rank-1's top halo, last owned
+    plane (nz-2) to rank+1's bottom halo — over torch.distributed point-to-point."""
+    os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port))
+    import sys
+    sys.path.insert(0, ROOT)
+    import torch
+    import oracle
+    from mdh_workloads import specs as S
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    try:
+        Z, Y, X, T = 11, 6, 7, 4
+        u0 = np.random.Generator(np.random.PCG64(3402)).random((Z, Y, X)).astype(np.float32)
+        lo, hi = S.z_slabs(Z, world)[rank]
+        nz = hi - lo + 2
+        spec = S.jacobi3d_sweep(nz, Y, X)
+        u = u0[lo - 1:hi + 1].astype(np.float64)
+        for _ in range(T):
+            u = oracle.stencil_sweeps(spec, u, 1)
+            t = torch.from_numpy(u)
+            reqs = []
+            if rank > 0:
+                reqs.append(dist.isend(t[1].contiguous(), rank - 1))
+                lo_recv = torch.empty_like(t[0])
+                reqs.append(dist.irecv(lo_recv, rank - 1))
+            if rank < world - 1:
+                reqs.append(dist.isend(t[nz - 2].contiguous(), rank + 1))
+                hi_recv = torch.empty_like(t[0])
+                reqs.append(dist.irecv(hi_recv, rank + 1))
+            for r in reqs:
+                r.wait()
+            if rank > 0:
+                u[0] = lo_recv.numpy()
+            if rank < world - 1:
+                u[nz - 1] = hi_recv.numpy()
+        gathered = [None] * world
+        dist.all_gather_object(gathered, (lo, hi, u[1:nz - 1]))
+        if rank == 0:
+            full = oracle.stencil_sweeps(S.jacobi3d_sweep(Z, Y, X), u0, T)
+            for glo, ghi, owned in gathered:
+                assert np.array_equal(owned, full[glo:ghi]), f"slab [{glo},{ghi}) differs"
+            q.put("ok")
+    except Exception as e:
+        q.put(f"rank {rank}: {type(e).__name__}: {e}")
+        raise
+    finally:
+        dist.destroy_process_group()
+
+
+@pytest.mark.parametrize("world", [2, 3])
+def test_stencil_sweeps_halo_exchange(world):
+    """F3: z-sharded Jacobi_3D time-stepping with a per-sweep halo exchange
+    reproduces the unsharded sweeps bit for bit (both fp64 oracle evaluations)."""
+    ctx = mp.get_context("spawn")
+    q = ctx.SimpleQueue()
+    port = _free_port()
+    procs = [ctx.Process(target=_sweeps_worker, args=(r, world, port, q)) for r in range(world)]
+    for pr in procs:
+        pr.start()
+    for pr in procs:
+        pr.join(180)
+    msgs = []
+    while not q.empty():
+        msgs.append(q.get())
+    assert all(pr.exitcode == 0 for pr in procs), msgs
+    assert "ok" in msgs, msgs

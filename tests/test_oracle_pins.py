@@ -369,3 +369,56 @@ def test_sampled_points_equal_full():
     lin, vals = oracle.evaluate_points(sp, ins, oracle.random_points(sp, 10))
     for b in range(3):
         assert np.array_equal(full[b].ravel()[lin[b]], vals[b])
+
+
+# ------------------------------------------------------------------ F3: stencil time-stepping
+def _j3d_numpy_sweeps(u0, sweeps):
+    """Independent formulation (numpy slicing, fp64) of reading C-34: interior update by the
+    seven shifted slabs of SURVEY §8(d) D-3 / reading C-16, boundary shell kept."""
+    w = S.J3D_WEIGHTS
+    u = u0.astype(np.float64).copy()
+    for _ in range(sweeps):
+        v = u.copy()
+        v[1:-1, 1:-1, 1:-1] = (w["c"] * u[1:-1, 1:-1, 1:-1]
+                               + w["xm"] * u[1:-1, 1:-1, :-2] + w["xp"] * u[1:-1, 1:-1, 2:]
+                               + w["ym"] * u[1:-1, :-2, 1:-1] + w["yp"] * u[1:-1, 2:, 1:-1]
+                               + w["zm"] * u[:-2, 1:-1, 1:-1] + w["zp"] * u[2:, 1:-1, 1:-1])
+        u = v
+    return u
+
+
+def test_stencil_sweeps_pins():
+    """oracle.stencil_sweeps (reading C-34) against: the single-sweep Jacobi_3D oracle (T=1,
+    interior), the numpy slicing formulation (T=3), the closed form c·(Σw)^T at points farther
+    than T from the boundary of a constant field, and the domain of dependence (a perturbation
+    at p changes nothing farther than T away after T sweeps)."""
+    Z, Y, X = 9, 10, 11
+    u0 = np.random.Generator(np.random.PCG64(3401)).random((Z, Y, X)).astype(np.float32)
+    sp = S.jacobi3d_sweep(Z, Y, X)
+    one = oracle.stencil_sweeps(sp, u0, 1)
+    ref1 = oracle.evaluate(S.jacobi3d(Z, Y, X), [u0])[0].reshape(Z - 2, Y - 2, X - 2)
+    assert np.array_equal(one[1:-1, 1:-1, 1:-1], ref1)
+    assert np.array_equal(one[0], u0[0].astype(np.float64)) and np.array_equal(one[:, :, -1], u0[:, :, -1].astype(np.float64))
+    three = oracle.stencil_sweeps(sp, u0, 3)
+    np.testing.assert_allclose(three, _j3d_numpy_sweeps(u0, 3), rtol=0, atol=1e-12)
+    # constant field: centre after T sweeps is c·(Σw)^T (distance to the shell > T)
+    c = 2.0
+    T = 3
+    const = oracle.stencil_sweeps(sp, np.full((Z, Y, X), c, np.float32), T)
+    sw = sum(S.J3D_WEIGHTS.values())
+    assert abs(const[4, 4, 5] - c * sw ** T) <= 1e-12
+    # domain of dependence (Manhattan distance ≤ T for the 7-point cross)
+    u1 = u0.copy()
+    u1[4, 5, 5] += 1.0
+    d = np.abs(oracle.stencil_sweeps(sp, u1, 2) - oracle.stencil_sweeps(sp, u0, 2))
+    zz, yy, xx = np.nonzero(d)
+    assert len(zz) and (np.abs(zz - 4) + np.abs(yy - 5) + np.abs(xx - 5)).max() <= 2
+
+
+def test_z_slabs_partition():
+    for Z, world in ((10, 1), (10, 3), (512, 8), (9, 7)):
+        sl = S.z_slabs(Z, world)
+        assert sl[0][0] == 1 and sl[-1][1] == Z - 1
+        assert all(a[1] == b[0] for a, b in zip(sl, sl[1:]))
+        sizes = [hi - lo for lo, hi in sl]
+        assert max(sizes) - min(sizes) <= 1 and min(sizes) >= 1
