@@ -80,6 +80,12 @@ def workload(name, world=1, rank=0):
         spec = S.jacobi3d(512, 512, 512)
         return dict(spec=spec, inputs=lambda: G.jacobi3d_inputs(512, 512, 512), work=4.0 * (512 ** 3 + 510 ** 3),
                     unit="GB/s", scale=1e9, bound="hbm", dtype="f32", desc="Jacobi3D 7-pt 512^3 fp32")
+    if name == "jacobi3d_sweeps8":
+        T = 8
+        spec = S.jacobi3d_sweep(512, 512, 512)
+        return dict(spec=spec, inputs=lambda: G.jacobi3d_inputs(512, 512, 512), work=T * 4.0 * (512 ** 3 + 510 ** 3),
+                    unit="GB/s", scale=1e9, bound="hbm", dtype="f32", sweeps=T,
+                    desc="Jacobi3D 7-pt 512^3 fp32, 8 sweeps u->v->u (mdh_stencil_sweeps; F3, reading C-34)")
     if name == "ccsd_bf16":
         spec = S.ccsd_sd1(24, 72, "bf16")
         out = 24 ** 3 * 72 ** 3
@@ -123,7 +129,7 @@ def workload(name, world=1, rank=0):
     raise SystemExit(f"unknown workload {name}")
 
 
-SUITE = ["dot_f32", "dot_i32", "dot_f32_2^28", "matvec_f32", "matvec_4096", "jacobi3d", "gaussian2d", "matmul_f32",
+SUITE = ["dot_f32", "dot_i32", "dot_f32_2^28", "matvec_f32", "matvec_4096", "jacobi3d", "jacobi3d_sweeps8", "gaussian2d", "matmul_f32",
          "matmul_bf16", "ccsd_bf16", "mcc_bf16", "mcc_caps_bf16", "prl_A", "prl_B", "prefix_sum_f32", "mbbs_f32"]
 
 
@@ -224,8 +230,14 @@ def run_mdh_workload(name, K, W, world, rank, dev, flush, pk, with_e2e=False, ch
     stream = torch.cuda.current_stream(dev)
     sh = stream.cuda_stream
 
-    def step():
-        plan(tin, outs, stream=sh, workspace_ptr=ws)
+    if w.get("sweeps"):                     # time-stepping: the output buffer is the second field
+        outs = [tin[0].clone()]
+
+        def step():
+            plan.stencil_sweeps(tin[0], outs[0], w["sweeps"], stream=sh, workspace_ptr=ws)
+    else:
+        def step():
+            plan(tin, outs, stream=sh, workspace_ptr=ws)
     for _ in range(W):
         step()
     torch.cuda.synchronize()

@@ -98,7 +98,9 @@ __device__ __forceinline__ void row6(const float* p, bool full, int64_t rem, flo
   }
 }
 
-template <bool VEC_IN, bool VEC_OUT>
+// VEC_OUT: 0 scalar stores; 1 two 8-byte stores (even output base); 2 odd output base
+// (e.g. the same-shape sweep of reading C-34, v[z+1,y+1,x+1]): scalar, 8-byte, scalar
+template <bool VEC_IN, int VEC_OUT>
 __global__ void __launch_bounds__(128) t1_j3d7_kernel(const __grid_constant__ J7Params P) {
   const int x0 = (blockIdx.x * 32 + threadIdx.x) * 4;
   const int y = blockIdx.y * 4 + threadIdx.y;
@@ -128,9 +130,13 @@ __global__ void __launch_bounds__(128) t1_j3d7_kernel(const __grid_constant__ J7
       acc = fmaf(P.wzp, rp[j + 1], acc);
       o[j] = acc;
     }
-    if (VEC_OUT && full) {
+    if (VEC_OUT == 1 && full) {
       reinterpret_cast<float2*>(po)[0] = make_float2(o[0], o[1]);
       reinterpret_cast<float2*>(po)[1] = make_float2(o[2], o[3]);
+    } else if (VEC_OUT == 2 && full) {
+      po[0] = o[0];
+      *reinterpret_cast<float2*>(po + 1) = make_float2(o[1], o[2]);
+      po[3] = o[3];
     } else {
 #pragma unroll
       for (int j = 0; j < 4; ++j)
@@ -401,12 +407,14 @@ static mdh_status launch_j3d7(const Plan& p, const void* const* in, void* const*
   P.zchunk = zc;
   const bool vin = (P.bc - 1) % 4 == 0 && P.Ly % 4 == 0 && P.Lz % 4 == 0;
   const bool vout = P.ob % 2 == 0 && P.oLy % 2 == 0 && P.oLz % 2 == 0;
+  const bool vodd = P.ob % 2 == 1 && P.oLy % 2 == 0 && P.oLz % 2 == 0;
   dim3 block(32, 4);
   dim3 grid((unsigned)((P.X + 127) / 128), (unsigned)((P.Y + 3) / 4), (unsigned)((P.Z + zc - 1) / zc));
-  if (vin && vout) t1_j3d7_kernel<true, true><<<grid, block, 0, st>>>(P);
-  else if (vin) t1_j3d7_kernel<true, false><<<grid, block, 0, st>>>(P);
-  else if (vout) t1_j3d7_kernel<false, true><<<grid, block, 0, st>>>(P);
-  else t1_j3d7_kernel<false, false><<<grid, block, 0, st>>>(P);
+  if (vin && vout) t1_j3d7_kernel<true, 1><<<grid, block, 0, st>>>(P);
+  else if (vin && vodd) t1_j3d7_kernel<true, 2><<<grid, block, 0, st>>>(P);
+  else if (vin) t1_j3d7_kernel<true, 0><<<grid, block, 0, st>>>(P);
+  else if (vout) t1_j3d7_kernel<false, 1><<<grid, block, 0, st>>>(P);
+  else t1_j3d7_kernel<false, 0><<<grid, block, 0, st>>>(P);
   return post_launch("t1_j3d7_kernel");
 }
 

@@ -34,10 +34,15 @@ def main():
         plan = Plan(w["spec"], force_tile=a.force_tile)
         tin = [to_device(x, b["dtype"], dev) for x, b in zip(w["inputs"](), w["spec"]["inputs"])]
         outs = plan.empty_outputs(dev)
+        if w.get("sweeps"):
+            outs = [tin[0].clone()]
+            step = lambda: plan.stencil_sweeps(tin[0], outs[0], w["sweeps"])
+        else:
+            step = lambda: plan(tin, outs)
         for _ in range(3):
-            plan(tin, outs)
+            step()
         torch.cuda.synchronize()
-        ts = sorted(bench.time_steps(lambda: plan(tin, outs), a.reps, torch.cuda.current_stream(), flush))
+        ts = sorted(bench.time_steps(step, a.reps, torch.cuda.current_stream(), flush))
         med = ts[len(ts) // 2]
         rl = bench.roofline(w, med, pk)
         print(json.dumps({"workload": name, "template": plan.template, "ms": round(med * 1e3, 4),
