@@ -219,10 +219,12 @@ mdh_status mdh_destroy(mdh_plan_t plan);
  * last owned planes of dst go to the neighbours' halo planes of their dst:
  *   - NCCL transport (nccl_comm from mdh_comm_init; one process per GPU): grouped
  *     ncclSend/ncclRecv on `cuda_stream`, any number of sweeps per call;
- *   - peer transport (nccl_comm NULL): device-to-device copies into peer_lo / peer_hi,
- *     the neighbours' halo planes (addresses this process can write: same device, P2P or
- *     CUDA-IPC mapped).  The caller orders the ranks' calls (one sweep per call, lock-step —
- *     e.g. virtual ranks on one stream).
+ *   - peer transport (nccl_comm NULL): the neighbours' halo planes peer_lo / peer_hi are
+ *     device addresses this process can write (same device, P2P or CUDA-IPC mapped); the
+ *     7-point kernel stores its first / last output plane into them itself (compute and
+ *     exchange in one kernel), other stencils are followed by device-to-device copies.
+ *     The caller orders the ranks' calls (one sweep per call, lock-step — e.g. virtual
+ *     ranks on one stream).
  * `workspace` as for mdh_execute.  On return *result_in_v = sweeps odd (the final field
  * is in v), else 0 (in u).  Errors: MDH_ERR_INVALID_ARG (bad plan shape, aliasing u/v,
  * sweeps < 0, missing transport, nz < 3), MDH_ERR_NCCL, MDH_ERR_CUDA.                  */

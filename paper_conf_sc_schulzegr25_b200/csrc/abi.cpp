@@ -333,6 +333,18 @@ mdh_status mdh_stencil_sweeps(mdh_plan_t plan, void* u, void* v, int32_t sweeps,
     const int s = t & 1, d = s ^ 1;
     const void* in[1] = {buf[s]};
     void* out[1] = {buf[d]};
+    if (world > 1 && !nccl) {
+      // peer transport: the 7-point kernel stores its first / last plane straight into the
+      // neighbours' halo planes as well (one kernel per sweep, no copies)
+      mdh::reset_launch_count();
+      mdh_status e = mdh::launch_t1_halo(p, buf[s], buf[d], rank > 0 ? halo->peer_lo[d] : nullptr,
+                                         rank < world - 1 ? halo->peer_hi[d] : nullptr, st);
+      if (e == MDH_OK) {
+        launches += mdh::launch_count();
+        continue;
+      }
+      if (e != MDH_ERR_UNSUPPORTED) return e;
+    }
     mdh_status e = mdh_execute(plan, in, out, workspace, workspace_bytes, cuda_stream);
     if (e != MDH_OK) return e;
     launches += mdh::launch_count();

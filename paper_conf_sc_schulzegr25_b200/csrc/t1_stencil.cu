@@ -83,6 +83,13 @@ struct J7Params {
   int64_t ob, oLy, oLz;    // output (x stride 1)
   int X, Y, Z, zchunk;
   float wc, wxm, wxp, wym, wyp, wzm, wzp;
+  // fused halo exchange (stencil time-stepping, reading C-34): the outputs of the first /
+  // last iteration plane are also stored into the lower / upper neighbour's halo plane
+  // (peer device memory: same GPU, NVLink P2P or CUDA-IPC mapped) at in-plane offset
+  // hbase + x + y·oLy; NULL = no neighbour
+  float* hlo;
+  float* hhi;
+  int64_t hbase;
 };
 
 template <bool VEC>
@@ -141,6 +148,19 @@ __global__ void __launch_bounds__(128) t1_j3d7_kernel(const __grid_constant__ J7
 #pragma unroll
       for (int j = 0; j < 4; ++j)
         if (x0 + j < P.X) po[j] = o[j];
+    }
+    float* ph = z == 0 ? P.hlo : (z == P.Z - 1 ? P.hhi : nullptr);
+    if (ph) {                      // this plane is also a neighbour's halo plane
+      ph += P.hbase + x0 + (int64_t)y * P.oLy;
+#pragma unroll
+      for (int j = 0; j < 4; ++j)
+        if (x0 + j < P.X) ph[j] = o[j];
+    }
+    if (P.hlo && P.hhi && P.Z == 1) {   // a one-plane slab feeds both neighbours
+      float* q = P.hhi + P.hbase + x0 + (int64_t)y * P.oLy;
+#pragma unroll
+      for (int j = 0; j < 4; ++j)
+        if (x0 + j < P.X) q[j] = o[j];
     }
 #pragma unroll
     for (int k = 0; k < 6; ++k) { rm[k] = r0[k]; r0[k] = rp[k]; }
@@ -382,9 +402,12 @@ mdh_status prepare_t1(Plan* p) {
   return MDH_OK;
 }
 
-static mdh_status launch_j3d7(const Plan& p, const void* const* in, void* const* out, cudaStream_t st) {
+static mdh_status launch_j3d7(const Plan& p, const void* const* in, void* const* out, cudaStream_t st,
+                              void* hlo = nullptr, void* hhi = nullptr) {
   J7Params P;
   memset(&P, 0, sizeof(P));
+  P.hlo = (float*)hlo;
+  P.hhi = (float*)hhi;
   const int dz = (int)p.auxi[0], dy = (int)p.auxi[1], dx = (int)p.auxi[2], c = (int)p.auxi[3];
   const Buf& B = p.in[0];
   const Access& O = p.out[0].acc[0];
@@ -396,6 +419,7 @@ static mdh_status launch_j3d7(const Plan& p, const void* const* in, void* const*
   P.ob = O.base;
   P.oLy = O.L[dy];
   P.oLz = O.L[dz];
+  P.hbase = O.base - O.L[dz];
   P.X = (int)p.size[dx];
   P.Y = (int)p.size[dy];
   P.Z = (int)p.size[dz];
@@ -416,6 +440,19 @@ static mdh_status launch_j3d7(const Plan& p, const void* const* in, void* const*
   else if (vout) t1_j3d7_kernel<false, 1><<<grid, block, 0, st>>>(P);
   else t1_j3d7_kernel<false, 0><<<grid, block, 0, st>>>(P);
   return post_launch("t1_j3d7_kernel");
+}
+
+// one sweep of a same-shape stencil plan with the halo stores fused into the 7-point
+// kernel (mdh_stencil_sweeps, peer transport); UNSUPPORTED when the plan does not run the
+// 7-point kernel or its first output plane is not buffer plane 1 (the caller then copies)
+mdh_status launch_t1_halo(const Plan& p, const void* in, void* out, void* hlo, void* hhi, cudaStream_t st) {
+  if (p.tmpl != T1_STENCIL || p.auxi.empty() || p.auxi[0] == -2) return MDH_ERR_UNSUPPORTED;
+  const Access& O = p.out[0].acc[0];
+  const int dz = (int)p.auxi[0];
+  if (O.L[dz] <= 0 || O.base < O.L[dz] || O.base >= 2 * O.L[dz]) return MDH_ERR_UNSUPPORTED;
+  const void* ins[1] = {in};
+  void* outs[1] = {out};
+  return launch_j3d7(p, ins, outs, st, hlo, hhi);
 }
 
 mdh_status launch_t1(const Plan& p, const void* const* in, void* const* out, void*, cudaStream_t st) {

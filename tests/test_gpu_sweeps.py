@@ -46,7 +46,9 @@ def test_sweeps_zsharded_virtual_ranks(world):
     """Slabs with one halo plane per side, a sweep per call in lock-step on one stream; after
     each sweep a rank's first / last owned plane is copied into the neighbours' halo planes
     (mdh_halo peer transport).  The owned planes equal the whole-domain GPU run bit for bit
-    (same per-point arithmetic) and the fp64 oracle within the scale-normalised 1e-4."""
+    (same per-point arithmetic) and the fp64 oracle within the scale-normalised 1e-4.  The
+    7-point kernel stores its first / last plane into the neighbours' halos itself (one
+    launch per sweep)."""
     import torch
     from paper_conf_sc_schulzegr25_b200 import Halo, Plan
     Z, Y, X, T = 23, 12, 40, 4
@@ -76,6 +78,7 @@ def test_sweeps_zsharded_virtual_ranks(world):
                     h.peer_hi[k] = bufs[r + 1][i].data_ptr()
             out = plans[r].stencil_sweeps(bufs[r][s], bufs[r][d], 1, halo=h)
             assert out is bufs[r][d]
+            assert Plan.last_launch_count() == 1       # halo stores fused into the sweep kernel
     torch.cuda.synchronize()
     whole_np = wres.cpu().numpy()
     ref, scale = _ref(Z, Y, X, u0, T)
