@@ -23,6 +23,8 @@
 #include <algorithm>
 #include <mutex>
 
+#include <type_traits>
+
 #include "kcommon.cuh"
 
 namespace mdh {
@@ -53,12 +55,21 @@ struct T6Params {
   void* z;        // V[Nc][T]
   void* loc;      // V[Nc][T]
   void* sums;     // V[Nc][nq]
+  // column fold (fp32, one pw dim, unit stride along the ps dim): row range split over
+  // S blocks × 8 threads; S > 1: per-split partials colpart[S][Nc·T] and a ticket per
+  // 128-column group (zero at rest); the last block folds the splits in order
+  int colS;
+  float* colpart;
+  unsigned* colcnt;
 };
 
 // K1 with the pw range split over threadIdx.y (blockDim.y contiguous sub-ranges, folded in
 // order through shared memory): 32 consecutive (c, t) points per block row keep loads
 // coalesced.  A single pw dim (MBBS's i) walks a plain stride, 8 loads in flight per
 // thread, added in index order.
+constexpr int T6_COL_SMAX = 32;
+constexpr int64_t T6_ROW_SMEM = 48 * 1024;   // rows up to this many bytes take t6_rowscan_kernel
+
 template <class V>
 __global__ void __launch_bounds__(1024) t6_fold_kernel(const __grid_constant__ T6Params P) {
   __shared__ V part[32][32];
@@ -129,6 +140,84 @@ __global__ void __launch_bounds__(1024) t6_fold_kernel(const __grid_constant__ T
   }
 }
 
+// K1 for MBBS-like shapes (few points, long pw range): each thread folds 4 consecutive
+// columns (one 16-byte load per row, 8 rows in flight) over its share of the rows; the
+// row range is split over blockIdx.y (S splits) × threadIdx.y (8), so S·(#column groups)
+// blocks fill the GPU even when the points alone cannot.  Fold order: rows ascending
+// inside a sub-range, sub-ranges (threadIdx.y, then blockIdx.y) ascending — fixed, so the
+// result is deterministic.
+__global__ void __launch_bounds__(256) t6_colfold_kernel(const __grid_constant__ T6Params P) {
+  __shared__ float4 part[8][32];
+  __shared__ int last;
+  const int64_t T = P.T;
+  const int64_t gpr = (T + 127) / 128;
+  const int64_t c = blockIdx.x / gpr, g = blockIdx.x % gpr;
+  const int64_t t = g * 128 + threadIdx.x * 4;
+  const int S = gridDim.y, s = blockIdx.y;
+  const int64_t npts = P.pwsize[0];
+  const int64_t nsub = (int64_t)S * 8, sub = (int64_t)s * 8 + threadIdx.y;
+  const int64_t per = (npts + nsub - 1) / nsub;
+  const int64_t r0 = min(npts, sub * per), r1 = min(npts, r0 + per);
+  float4 acc = make_float4(0.f, 0.f, 0.f, 0.f);
+  if (t < T && r0 < r1) {
+    int64_t off = P.base[0] + P.Lt[0] * t, rem = c;
+    for (int q = P.nrowd - 1; q >= 0; --q) {
+      const int64_t v = rem % P.rowsize[q];
+      rem /= P.rowsize[q];
+      off += P.Lrow[0][q] * v;
+    }
+    const int64_t L = P.Lpw[0][0];
+    const float* x = (const float*)P.ptr[0] + off + L * r0;
+    acc = __ldg(reinterpret_cast<const float4*>(x));
+    x += L;
+    int64_t r = r0 + 1;
+    for (; r + 8 <= r1; r += 8, x += 8 * L) {
+      float4 y[8];
+#pragma unroll
+      for (int u = 0; u < 8; ++u) y[u] = __ldg(reinterpret_cast<const float4*>(x + u * L));
+#pragma unroll
+      for (int u = 0; u < 8; ++u) { acc.x += y[u].x; acc.y += y[u].y; acc.z += y[u].z; acc.w += y[u].w; }
+    }
+    for (; r < r1; ++r, x += L) {
+      const float4 y = __ldg(reinterpret_cast<const float4*>(x));
+      acc.x += y.x; acc.y += y.y; acc.z += y.z; acc.w += y.w;
+    }
+  }
+  part[threadIdx.y][threadIdx.x] = acc;
+  __syncthreads();
+  const int64_t e = c * T + t;
+  if (threadIdx.y == 0) {
+    float4 b = part[0][threadIdx.x];
+    for (int y = 1; y < 8; ++y) {
+      const float4 q = part[y][threadIdx.x];
+      b.x += q.x; b.y += q.y; b.z += q.z; b.w += q.w;
+    }
+    if (t < T) {
+      if (S == 1) *reinterpret_cast<float4*>((float*)P.z + e) = b;
+      else *reinterpret_cast<float4*>(P.colpart + (int64_t)s * P.Nc * T + e) = b;
+    }
+  }
+  if (S > 1) {
+    __threadfence();
+    __syncthreads();
+    if (threadIdx.x == 0 && threadIdx.y == 0) last = atomicAdd(P.colcnt + blockIdx.x, 1u) == (unsigned)(S - 1);
+    __syncthreads();
+    if (!last) return;
+    if (threadIdx.y == 0) {
+      __threadfence();
+      if (t < T) {
+        float4 b = __ldcg(reinterpret_cast<const float4*>(P.colpart + e));
+        for (int k = 1; k < S; ++k) {
+          const float4 q = __ldcg(reinterpret_cast<const float4*>(P.colpart + (int64_t)k * P.Nc * T + e));
+          b.x += q.x; b.y += q.y; b.z += q.z; b.w += q.w;
+        }
+        *reinterpret_cast<float4*>((float*)P.z + e) = b;
+      }
+      if (threadIdx.x == 0) P.colcnt[blockIdx.x] = 0u;   // back to rest for the next execute
+    }
+  }
+}
+
 __device__ __forceinline__ int64_t t6_out_offset(const T6Params& P, int64_t c, int64_t t) {
   int64_t o = P.obase + P.oLt * t, rem = c;
   for (int q = P.nrowd - 1; q >= 0; --q) {
@@ -137,6 +226,51 @@ __device__ __forceinline__ int64_t t6_out_offset(const T6Params& P, int64_t c, i
     o += P.orowL[q] * v;
   }
   return o;
+}
+
+// Inclusive scan of short rows (T ≤ T6_ROW_MAX) of the fold result z, one block of 1024
+// threads per row: the row is staged in shared memory by coalesced loads, each thread
+// scans a segment of ⌈T/1024⌉ consecutive elements, segment totals are scanned by warp
+// shuffles (lane order) and then across the 32 warps (warp order) — a fixed association,
+// deterministic — and the result leaves through out_view with coalesced stores.
+template <class V>
+__global__ void __launch_bounds__(1024) t6_rowscan_kernel(const __grid_constant__ T6Params P) {
+  extern __shared__ __align__(16) unsigned char t6rs_raw[];
+  V* zs = reinterpret_cast<V*>(t6rs_raw);
+  __shared__ V wtot[32];
+  const int64_t c = blockIdx.x, T = P.T;
+  const int tid = threadIdx.x, lane = tid & 31, wid = tid >> 5;
+  const V* zr = (const V*)P.z + c * T;
+  for (int64_t k = tid; k < T; k += 1024) zs[k] = zr[k];
+  __syncthreads();
+  const int64_t seg = (T + 1023) / 1024;
+  const int64_t a0 = min(T, tid * seg), a1 = min(T, a0 + seg);
+  V sum = (V)0;
+  for (int64_t k = a0; k < a1; ++k) sum = Arith<V>::add(sum, zs[k]);
+  V incl = sum;                                   // inclusive scan over the lanes
+#pragma unroll
+  for (int o = 1; o < 32; o <<= 1) {
+    const V y = __shfl_up_sync(0xffffffffu, incl, o);
+    if (lane >= o) incl = Arith<V>::add(y, incl);
+  }
+  V excl = __shfl_up_sync(0xffffffffu, incl, 1);
+  if (lane == 0) excl = (V)0;
+  if (lane == 31) wtot[wid] = incl;
+  __syncthreads();
+  if (wid == 0) {
+    V w = wtot[lane];
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+      const V y = __shfl_up_sync(0xffffffffu, w, o);
+      if (lane >= o) w = Arith<V>::add(y, w);
+    }
+    wtot[lane] = w;                               // inclusive over warps
+  }
+  __syncthreads();
+  V run = wid > 0 ? Arith<V>::add(wtot[wid - 1], excl) : excl;   // exclusive prefix of the segment
+  for (int64_t k = a0; k < a1; ++k) { run = Arith<V>::add(run, zs[k]); zs[k] = run; }
+  __syncthreads();
+  for (int64_t k = tid; k < T; k += 1024) store_as<V>(P.out, P.odt, t6_out_offset(P, c, k), zs[k]);
 }
 
 // block inclusive scan of one chunk; writes either the final output (single chunk) or the
@@ -763,6 +897,18 @@ mdh_status prepare_t6(Plan* p) {
   }
   p->auxi.clear();
   p->ws_kernel = al((size_t)Nc * T * vs) + (nq > 1 ? al((size_t)Nc * T * vs) + al((size_t)Nc * nq * vs) : 0);
+  // column fold (t6_colfold_kernel): fp32, one pw dim, the ps dim unit-stride, few points
+  // (≤ 2^20) — room for T6_COL_SMAX split partials and the per-group tickets
+  int npw = 0;                            // pw dims (p->red also lists the ps dim)
+  for (int t = 0; t < p->nred; ++t) npw += p->red[t] != dps;
+  const bool col = npw == 1 && p->f == MDH_F_IDENTITY && p->n_in_acc == 1 && p->in[0].dtype == MDH_F32 &&
+                   p->compute == MDH_F32 && p->in[0].acc[0].L[dps] == 1 && T % 4 == 0 && Nc * T <= (1 << 20);
+  if (col) {
+    p->auxi.assign(2, 0);
+    p->auxi[0] = -2;                      // marker: column fold eligible (launch re-checks alignment)
+    p->auxi[1] = (int64_t)p->ws_kernel;   // offset of the split partials
+    p->ws_kernel += al((size_t)T6_COL_SMAX * Nc * T * 4) + al((size_t)Nc * ((T + 127) / 128) * 4);
+  }
   return MDH_OK;
 }
 
@@ -814,10 +960,21 @@ static mdh_status launch_typed(const T6Params& P, cudaStream_t st) {
     // the GPU (MBBS: 8192 points × 8192 rows), else 8
     int64_t npts = 1;
     for (int q = 0; q < P.npw; ++q) npts *= P.pwsize[q];
-    const int Y = (npts >= 1024 && total < 148LL * 2048) ? 32 : 8;
-    const unsigned gf = (unsigned)std::max<int64_t>(1, std::min<int64_t>((total + 31) / 32, 148LL * 64));
-    t6_fold_kernel<V><<<gf, dim3(32, Y), 0, st>>>(P);
-    MDH_TRY(post_launch("t6_fold_kernel"));
+    if (std::is_same<V, float>::value && P.colS > 0) {
+      const unsigned groups = (unsigned)(P.Nc * ((P.T + 127) / 128));
+      t6_colfold_kernel<<<dim3(groups, (unsigned)P.colS), dim3(32, 8), 0, st>>>(P);
+      MDH_TRY(post_launch("t6_colfold_kernel"));
+    } else {
+      const int Y = (npts >= 1024 && total < 148LL * 2048) ? 32 : 8;
+      const unsigned gf = (unsigned)std::max<int64_t>(1, std::min<int64_t>((total + 31) / 32, 148LL * 64));
+      t6_fold_kernel<V><<<gf, dim3(32, Y), 0, st>>>(P);
+      MDH_TRY(post_launch("t6_fold_kernel"));
+    }
+  }
+  if (!P.direct && P.T * (int64_t)sizeof(V) <= T6_ROW_SMEM && P.Nc <= INT32_MAX) {
+    // short rows: one single-block scan per row instead of chunk scan + totals + fix-up
+    t6_rowscan_kernel<V><<<(unsigned)P.Nc, 1024, (size_t)P.T * sizeof(V), st>>>(P);
+    return post_launch("t6_rowscan_kernel");
   }
   if (P.Nc > 65535) { set_error("T6: too many rows"); return MDH_ERR_UNSUPPORTED; }
   dim3 grid((unsigned)P.nq, (unsigned)P.Nc);
@@ -882,7 +1039,7 @@ mdh_status launch_t6(const Plan& p, const void* const* in, void* const* out, voi
   const int64_t vs = vsize(p.compute);
   auto al = [](size_t x) { return (x + 255) / 256 * 256; };
   char* w = (char*)ws;
-  if (!p.auxi.empty() && p.auxi[0] < 0) {          // streaming scan (prepare_t6)
+  if (p.auxi.size() == 1 && p.auxi[0] == -1) {    // streaming scan (prepare_t6)
     P.loc = w;                                      // header: epoch, done counter
     P.z = w + 256;                                  // tagged CTA totals [8][G]
     switch (p.compute) {
@@ -894,7 +1051,8 @@ mdh_status launch_t6(const Plan& p, const void* const* in, void* const* out, voi
       default: set_error("T6: unsupported type"); return MDH_ERR_UNSUPPORTED;
     }
   }
-  if (!p.auxi.empty()) {                  // segmented single-pass scan (prepare_t6)
+  const bool colfold = p.auxi.size() == 2 && p.auxi[0] == -2;
+  if (!p.auxi.empty() && !colfold) {      // segmented single-pass scan (prepare_t6)
     P.nq = p.auxi[0];
     switch (p.compute) {
       case MDH_F32: return launch_seg<float>(P, w, st);
@@ -908,6 +1066,24 @@ mdh_status launch_t6(const Plan& p, const void* const* in, void* const* out, voi
   P.z = w;
   P.loc = w + al((size_t)P.Nc * P.T * vs);
   P.sums = (char*)P.loc + al((size_t)P.Nc * P.T * vs);
+  if (colfold && !P.direct) {
+    // 16-byte loads need every point's first element 16-byte aligned
+    bool aligned = (uintptr_t)P.ptr[0] % 16 == 0 && P.base[0] % 4 == 0;
+    for (int q = 0; q < P.nrowd; ++q) aligned &= P.Lrow[0][q] % 4 == 0;
+    aligned &= P.Lpw[0][0] % 4 == 0;
+    if (aligned) {
+      int dev = 0, sms = 148;
+      MDH_CUDA(cudaGetDevice(&dev));
+      MDH_CUDA(cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev));
+      const int64_t groups = P.Nc * ((P.T + 127) / 128);
+      // splits so that the blocks fill 8 × 256 threads per SM, rows per thread ≥ 32
+      int64_t S = std::max<int64_t>(1, (int64_t)sms * 8 / std::max<int64_t>(1, groups));
+      S = std::min<int64_t>({S, (int64_t)T6_COL_SMAX, std::max<int64_t>(1, P.pwsize[0] / 256)});
+      P.colS = (int)S;
+      P.colpart = (float*)(w + p.auxi[1]);
+      P.colcnt = (unsigned*)(w + p.auxi[1] + al((size_t)T6_COL_SMAX * P.Nc * P.T * 4));
+    }
+  }
   switch (p.compute) {
     case MDH_F32: return launch_typed<float>(P, st);
     case MDH_F64: return launch_typed<double>(P, st);

@@ -98,8 +98,11 @@ def test_gpu_single_pass_scan(shape, dt, tile):
 
 
 @gpu
-@pytest.mark.parametrize("IJ", [(64, 37), (1000, 5000), (4096, 8192)])
+@pytest.mark.parametrize("IJ", [(64, 37), (1000, 5000), (4096, 8192), (8192, 8192), (300, 1000), (40, 64)])
 def test_gpu_mbbs(IJ):
+    """MBBS on T6; shapes with J % 4 == 0 take the column-fold K1 (16-byte column loads,
+    the row range split over blocks, ordered ticket fold; ragged last column group for
+    J = 1000).  Run twice on one plan: tickets back at rest, results bit-identical."""
     from gpu_util import assert_close_full, run_gpu
     spec = S.mbbs(*IJ)
     x = G.gen_inputs(spec, 6200, "positive")
@@ -110,6 +113,8 @@ def test_gpu_mbbs(IJ):
     else:   # closed form R[j] = Σ_{j'≤j} Σ_i X[i,j'] (pinned against the oracle above)
         ref = np.cumsum(x[0].astype(np.float64).sum(axis=0))
         assert np.max(np.abs(got[0] - ref) / ref) <= 1e-4
+    got2, _ = run_gpu(spec, x, plan=p)
+    assert np.array_equal(got[0], got2[0])
 
 
 @gpu
