@@ -1702,11 +1702,11 @@ mdh_status prepare_t4(Plan* p) {
       P.num_tiles = ((P.tiles_m + 1) / 2) * P.tiles_n;
     } else if (c.N > 256 && p->tiles.bn != 256 &&
                (p->tiles.bn == 512 || icp.a_im2col ||
-                (int64_t)P.tiles_m * ((c.N + 511) / 512) >= 2 * std::max(1, plan_sms(p) / 2))) {
+                (int64_t)P.tiles_m * ((c.N + 511) / 512) >= std::max(1, plan_sms(p) / 2))) {
       // wide pair tiles 256×512: A is requested once per 8.4 MFLOP instead of
-      // per 4.2.  Auto for an im2col A (MCC conv5_1: 67.6 vs 71.8 µs) and for GEMMs with at
-      // least two waves of wide tiles (8192³: 1461 vs 1321 TFLOP/s; at 4096³, 1.7 waves, the
-      // narrow tiles' overlapped epilogues win: 114.7 vs 115.7 µs); tile knob bn=256|512
+      // per 4.2.  Auto for an im2col A (MCC conv5_1) and for GEMMs with at least one full
+      // wave of wide tiles (tools/sweep_tiles.py, whole tiles: 4096³ 106.6 vs 116.7 µs, 8192³
+      // 717.7 vs 840.7 µs; 2048³, 32 wide tiles: narrow 24.6 vs 35.7 µs); tile knob bn=256|512
       s->nw = 512;
       P.tiles_n = (int)((c.N + 511) / 512);
       P.num_tiles = P.tiles_m * P.tiles_n;
@@ -2035,7 +2035,13 @@ mdh_status launch_t4(const Plan& p, const void* const* in, void* const* out, voi
     P.nfull = T;
     P.sk_pairs = 0;
     P.sk_w = 0;
-    if (T % C != 0 && p.tiles.split != 1) {
+    // auto: stream-K only for a single partial wave of deep tiles (MCC conv5_1: 49 wide tiles
+    // of 72 k-blocks on 74 pairs, 63.5 vs 66.3 µs); with more waves or shallow tiles the
+    // fixups cost more than the balance gains (4096³ wide 108.8 vs 106.6 µs, 2048³ narrow
+    // 32.7 vs 24.6 µs; tools/sweep_tiles.py).  Tile knob split=1 never, split≥2 whenever
+    // the last wave is partial.
+    const bool sk_auto = T < C && P.num_kb >= 64;
+    if (T % C != 0 && (p.tiles.split >= 2 || (p.tiles.split == 0 && sk_auto))) {
       // every complete wave runs whole tiles (their epilogues overlap later MMAs); only the
       // partial last wave is spread over all pairs, so few outputs are written at the end
       const int nfull = R * C;

@@ -465,9 +465,9 @@ def test_t4_split_tail_1sm(shape, tile, out):
         assert_close_points(spec, x, got, 1e-2, n=20000, kind="rel")
 
 
-@pytest.mark.parametrize("shape,tile,kind", [((512, 512, 8192), None, "full"),       # 4 tiles, ~16 pairs each
-                                             ((2500, 2000, 1000), None, "points"),   # ragged, 80 tiles / 74 pairs
-                                             ((4096, 4096, 4096), None, "points"),   # 2 data-parallel waves + SK
+@pytest.mark.parametrize("shape,tile,kind", [((512, 512, 8192), "split=2", "full"),  # 4 tiles, ~16 pairs each
+                                             ((2500, 2000, 1000), "bn=256,split=2", "points"),   # ragged, 80 tiles / 74 pairs
+                                             ((4096, 4096, 4096), "bn=256,split=2", "points"),   # 3 whole waves + SK
                                              ((1024, 768, 640), "split=1", "full"),   # whole tiles only
                                              ((700, 1000, 1000), "cluster=4", "full"),  # odd row tiles: an idle pair
                                              ((2500, 2000, 1000), "cluster=4", "points"),  # 4-CTA clusters
@@ -475,7 +475,8 @@ def test_t4_split_tail_1sm(shape, tile, out):
                                              ((2500, 2000, 1000), "bn=512", "points"),
                                              ((4096, 4096, 4096), "bn=512", "points")])
 def test_t4_stream_k(shape, tile, kind):
-    """2-SM stream-K hybrid: whole-tile waves, then each cluster's even share of the remaining
+    """2-SM stream-K hybrid (forced with split≥2 where the auto rule / tile table would pick
+    whole tiles): whole-tile waves, then each cluster's even share of the remaining
     (tile, k-block) space; producers publish coalesced fp32 partials, the finisher (the one
     holding k = 0) adds them in k order.  Single pairs (default) and 4-CTA clusters
     (cluster=4: two pairs sharing B by TMA multicast; with an odd number of 256-row tiles

@@ -32,6 +32,16 @@ def cases():
          [f"zchunk={z}" for z in (8, 16, 32, 64, 128, 255, 510)]),
         ("prl_B", lambda: (S.prl(1 << 14, 1 << 20), G.prl_inputs(1 << 14, 1 << 20)),
          [f"split={s}" for s in (8, 16, 32, 37, 48, 64)]),
+        # T4 2-SM: pair-tile width (256 / 512) × whole tiles vs stream-K for the last wave
+        ("t4_mm_bf16_4096", lambda: (S.matmul(4096, 4096, 4096, "bf16"), G.matmul_inputs(4096, 4096, 4096, "bf16", "signed")),
+         ["bn=256", "bn=512", "bn=256,split=1", "bn=512,split=1"]),
+        ("t4_mm_bf16_8192", lambda: (S.matmul(8192, 8192, 8192, "bf16"), G.matmul_inputs(8192, 8192, 8192, "bf16", "signed")),
+         ["bn=256", "bn=512", "bn=256,split=1", "bn=512,split=1"]),
+        ("t4_mm_bf16_2048", lambda: (S.matmul(2048, 2048, 2048, "bf16"), G.matmul_inputs(2048, 2048, 2048, "bf16", "signed")),
+         ["bn=256", "bn=512", "bn=256,split=1", "bn=512,split=1"]),
+        ("t4_mcc_bf16_conv5_1", lambda: (S.mcc(256, 7, 7, 512, 3, 3, 512, "bf16"),
+                                         G.mcc_inputs(S.mcc(256, 7, 7, 512, 3, 3, 512, "bf16"))),
+         ["bn=256", "bn=512", "bn=256,split=1", "bn=512,split=1"]),
         ("mcc_f32_n1", lambda: (S.mcc(1, 7, 7, 512, 3, 3, 512, "f32"),
                                 G.mcc_inputs(S.mcc(1, 7, 7, 512, 3, 3, 512, "f32"))),
          [f"split={s}" for s in (1, 8, 16, 32, 64, 72)]),
