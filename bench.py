@@ -96,6 +96,10 @@ def workload(name, world=1, rank=0):
         spec = S.mcc(256, 7, 7, 512, 3, 3, 512, "bf16")
         return dict(spec=spec, inputs=lambda: G.mcc_inputs(spec), work=2.0 * 256 * 49 * 512 * 4608, unit="TFLOP/s",
                     scale=1e12, bound="tensor", dtype="bf16", desc="MCC ResNet-50 conv5_1 3x3/s2 N=256 bf16")
+    if name == "mcc_bf16_n1":
+        spec = S.mcc(1, 7, 7, 512, 3, 3, 512, "bf16")
+        return dict(spec=spec, inputs=lambda: G.mcc_inputs(spec), work=2.0 * 49 * 512 * 4608, unit="TFLOP/s",
+                    scale=1e12, bound="tensor", dtype="bf16", desc="MCC ResNet-50 conv5_1 3x3/s2 N=1 bf16 (the paper's batch)")
     if name == "gaussian2d":
         I = J = 4096
         spec = S.gaussian2d(I, J)
@@ -130,7 +134,7 @@ def workload(name, world=1, rank=0):
 
 
 SUITE = ["dot_f32", "dot_i32", "dot_f32_2^28", "matvec_f32", "matvec_4096", "jacobi3d", "jacobi3d_sweeps8", "gaussian2d", "matmul_f32",
-         "matmul_bf16", "ccsd_bf16", "mcc_bf16", "mcc_caps_bf16", "prl_A", "prl_B", "prefix_sum_f32", "mbbs_f32"]
+         "matmul_bf16", "ccsd_bf16", "mcc_bf16", "mcc_bf16_n1", "mcc_caps_bf16", "prl_A", "prl_B", "prefix_sum_f32", "mbbs_f32"]
 
 
 def roofline(w, seconds, pk):

@@ -106,6 +106,8 @@ struct Params {
   unsigned long long* trace;
   int trace_n;                      // units the trace buffer holds
   int c_vec4;                       // row-major C with ldc, cbase ≡ 0 mod 4 and a 16-byte base
+  int xfold;                        // 1-SM split-K over few tiles: every split writes its partial,
+                                    // t4_xfold_kernel folds them in split order afterwards
 };
 
 constexpr int AG_WARPS = 4, AG_THREADS = AG_WARPS * 32, KOFF_MAX = 2048;
@@ -667,7 +669,7 @@ __global__ void __launch_bounds__(AG ? THREADS + AG_THREADS : THREADS, 1)
       // p_0 + … + p_{S-2} + own in split order before the store
       const bool split = slot >= 0;
       const int ti = split ? slot / P.ssplit : 0;
-      const bool last = split && slot % P.ssplit == P.ssplit - 1;
+      const bool last = split && !P.xfold && slot % P.ssplit == P.ssplit - 1;
       unsigned* cnt = P.tail_cnt + 2 * ti;
       const int64_t prel = (int64_t)row * BN + half * (BN / 2);
       float* prow = (split && !last) ? P.part + (int64_t)slot * (BM * BN) + prel : nullptr;
@@ -765,7 +767,7 @@ __global__ void __launch_bounds__(AG ? THREADS + AG_THREADS : THREADS, 1)
           }
         }
       }
-      if (split && !last) {            // publish this warp's part of the partial tile
+      if (split && !last && !P.xfold) {   // publish this warp's part of the partial tile
         __threadfence();
         __syncwarp();
         if (lane == 0) atomicAdd(cnt, 1u);
@@ -1258,6 +1260,39 @@ __global__ void __cluster_dims__(CL, 1, 1) __launch_bounds__(THREADS, 1)
   if (P.trace && threadIdx.x == 0 && pair_gid < 256) P.trace[8 * P.trace_n + 2 * pair_gid + 1 + rank * 512] = gtimer();
 }
 
+// Few-tile split-K (1-SM kernel, P.xfold): S splits of each of the T tiles wrote dense
+// fp32 partial tiles [128][256]; fold them in split order (deterministic) across the whole
+// GPU and write through out_view (row-major or the offset tables; fp32 or bf16).
+__global__ void __launch_bounds__(256) t4_xfold_kernel(const __grid_constant__ Params P) {
+  constexpr int64_t PT = (int64_t)BM * BN;
+  const int64_t per_tile = PT / 4;
+  const int64_t total = (int64_t)(P.nunits / P.ssplit) * per_tile;
+  for (int64_t e = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; e < total; e += (int64_t)gridDim.x * blockDim.x) {
+    const int64_t ti = e / per_tile, q = e % per_tile;
+    const int r = (int)(q / (BN / 4)), c4 = (int)(q % (BN / 4)) * 4;
+    const float* src = P.part + ti * P.ssplit * PT + (int64_t)r * BN + c4;
+    float4 a = __ldcg(reinterpret_cast<const float4*>(src));
+    for (int sp = 1; sp < P.ssplit; ++sp) {
+      const float4 b = __ldcg(reinterpret_cast<const float4*>(src + sp * PT));
+      a.x += b.x; a.y += b.y; a.z += b.z; a.w += b.w;
+    }
+    int mb, nb;
+    t_decode(P, P.nfull + (int)ti, &mb, &nb);
+    const int64_t m = (int64_t)mb * BM + r;
+    if (m >= P.M) continue;
+    const int64_t row = P.cbase + (P.c_rowmajor ? m * P.ldc : P.cM[m]);
+    const float v[4] = {a.x, a.y, a.z, a.w};
+#pragma unroll
+    for (int j = 0; j < 4; ++j) {
+      const int64_t n = (int64_t)nb * BN + c4 + j;
+      if (n >= P.N) break;
+      const int64_t o = row + (P.c_rowmajor ? n : P.cN[n]);
+      if (P.out_bf16) ((__nv_bfloat16*)P.C)[o] = __float2bfloat16_rn(v[j]);
+      else P.C[o] = v[j];
+    }
+  }
+}
+
 constexpr int SK_MAX_PAIRS = 74;     // stream-K partial slots reserved in the workspace (2-SM path)
 constexpr int SK_MIN_SEG = 8;        // shortest stream-K range per pair, in 64-deep k-blocks
 constexpr int MAX_TAIL_UNITS1 = 296; // 1-SM path: bound on tail units (partials sized per plan)
@@ -1726,7 +1761,26 @@ mdh_status prepare_t4(Plan* p) {
     }
     const int T = P.num_tiles, C = std::max(1, std::min(T, sms)), R = T / C, Tr = T - R * C;
     int S = 1;
-    if (Tr > 0) {
+    if (4 * T <= sms && P.num_kb >= 16 && p->tiles.split != 1) {
+      // few tiles, deep K (MCC conv5_1 at the paper's N = 1: 2 tiles × 72 k-blocks): split
+      // every tile along K over the idle SMs, all splits write partials, and a separate
+      // grid-wide fold (t4_xfold_kernel) adds them in split order
+      S = std::min({sms / T, P.num_kb / 4, t4::MAX_TAIL_UNITS1 / T});
+      if (p->tiles.split > 1) S = std::min(S, p->tiles.split);
+      if (S >= 2) {
+        P.xfold = 1;
+        P.sched = 0;
+        P.nfull = 0;
+        P.ssplit = S;
+        P.nunits = T * S;
+        ws = (ws + 255) / 256 * 256;
+        s->tail_off = ws;
+        ws += (size_t)T * S * t4::BM * t4::BN * sizeof(float) + 2 * (size_t)T * sizeof(unsigned) + 256;
+        s->tail_parts = T * S;
+        s->grid1 = std::min(T * S, sms);
+        S = 1;                                   // (the tail logic below is skipped)
+      }
+    } else if (Tr > 0) {
       const int cap = std::min({C / Tr, P.num_kb / 4, t4::MAX_TAIL_UNITS1 / Tr});
       if (p->tiles.split > 1) S = std::min(p->tiles.split, cap);
       // (no automatic split: on MCC conv5_1 split 2/3/4 measured 84/92/92 µs vs 84 whole)
@@ -1884,6 +1938,14 @@ static mdh_status make_map(CUtensorMap* map, const void* base, int64_t inner, in
                   CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
   if (r != CUDA_SUCCESS) { set_error("cuTensorMapEncodeTiled failed (%d)", (int)r); return MDH_ERR_CUDA; }
   return MDH_OK;
+}
+
+static mdh_status launch_xfold(const t4::Params& P, int sms, cudaStream_t st) {
+  if (!P.xfold) return MDH_OK;
+  const int64_t work = (int64_t)(P.nunits / P.ssplit) * t4::BM * t4::BN / 4;
+  const unsigned g = (unsigned)std::max<int64_t>(1, std::min<int64_t>((work + 255) / 256, (int64_t)sms * 8));
+  t4::t4_xfold_kernel<<<g, 256, 0, st>>>(P);
+  return post_launch("t4_xfold_kernel");
 }
 
 static mdh_status run_permute(const t4::Layout2D& L, const uint16_t* src, char* ws, const int64_t* offMN,
@@ -2097,7 +2159,8 @@ mdh_status launch_t4(const Plan& p, const void* const* in, void* const* out, voi
     else if (epi2) t4::gemm_kernel<2, true, true><<<grid, TG, t4::SMEM_AG_BYTES, st>>>(ma, mb, P);
     else if (!P.out_bf16) t4::gemm_kernel<1, false, true><<<grid, TG, t4::SMEM_AG_BYTES, st>>>(ma, mb, P);
     else t4::gemm_kernel<1, true, true><<<grid, TG, t4::SMEM_AG_BYTES, st>>>(ma, mb, P);
-    return post_launch("t4_gemm_kernel_ag");
+    MDH_TRY(post_launch("t4_gemm_kernel_ag"));
+    return launch_xfold(P, sms, st);
   }
   if (s->epi == 3 && (uintptr_t)P.C % 16 == 0) {
     t4::gemm_kernel<3, false><<<grid, t4::THREADS, s->smem3, st>>>(ma, mb, P);
@@ -2112,7 +2175,8 @@ mdh_status launch_t4(const Plan& p, const void* const* in, void* const* out, voi
   else if (epi2) t4::gemm_kernel<2, true><<<grid, t4::THREADS, t4::SMEM_BYTES, st>>>(ma, mb, P);
   else if (!P.out_bf16) t4::gemm_kernel<1, false><<<grid, t4::THREADS, t4::SMEM_BYTES, st>>>(ma, mb, P);
   else t4::gemm_kernel<1, true><<<grid, t4::THREADS, t4::SMEM_BYTES, st>>>(ma, mb, P);
-  return post_launch("t4_gemm_kernel");
+  MDH_TRY(post_launch("t4_gemm_kernel"));
+  return launch_xfold(P, sms, st);
 }
 
 }  // namespace mdh

@@ -505,6 +505,21 @@ def test_t4_stream_k(shape, tile, kind):
         assert np.all(got[0] == float(K))
 
 
+@pytest.mark.parametrize("shape,out", [((100, 300, 4096), "f32"), ((100, 300, 4096), "bf16"), ((64, 512, 2048), "f32")])
+def test_t4_few_tile_splitk(shape, out):
+    """1-SM kernel with few tiles and a deep K (as MCC conv5_1 at N = 1): every tile is split
+    along K over the idle SMs, all splits write partials, t4_xfold_kernel folds them in split
+    order; ragged M / N, fp32 and bf16 outputs; deterministic across runs."""
+    M, N, K = shape
+    spec = S.matmul(M, N, K, "bf16", out_dtype=out)
+    x = G.matmul_inputs(M, N, K, "bf16", "positive")
+    got, p = run_gpu(spec, x)
+    assert not p.describe()["t4_variant"] & 8
+    assert_close_full(spec, x, got, 1e-2, kind="rel")
+    got2, _ = run_gpu(spec, x, plan=p)
+    assert np.array_equal(got[0], got2[0])
+
+
 def test_mcc_bf16_config_sampled():
     spec = S.mcc(256, 7, 7, 512, 3, 3, 512, "bf16")
     x = G.mcc_inputs(spec)
