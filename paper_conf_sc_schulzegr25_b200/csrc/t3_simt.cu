@@ -160,43 +160,52 @@ struct T3Lin {
 // run (no short-scoreboard stall on the LDS results)
 template <bool FP>
 __global__ void __launch_bounds__(256, FP ? 1 : 2) t3_linear_kernel(const __grid_constant__ T3Lin P) {
-  __shared__ __align__(16) float As[2][8][128 + 4];
-  __shared__ __align__(16) float Bs[2][8][128];
+  constexpr int KB = FP ? 16 : 8;                 // k-block (FP: half as many barriers)
+  constexpr int H = KB / 8;                        // 8-deep slices per k-block
+  __shared__ __align__(16) float As[2][KB][128 + 4];
+  __shared__ __align__(16) float Bs[2][KB][128];
   const int tid = threadIdx.x, tx = tid & 15, ty = tid >> 4;
   const int m0 = blockIdx.y * 128, n0 = blockIdx.x * 128;
-  const int am = tid >> 1, ak = (tid & 1) * 4;      // A: row am, 4 consecutive k
-  const int bk = tid >> 5, bn = (tid & 31) * 4;     // B: row bk, 4 consecutive n
+  const int am = tid >> 1, ak = (tid & 1) * 4;      // A: row am, 4 consecutive k (+8h)
+  const int bk = tid >> 5, bn = (tid & 31) * 4;     // B: row bk (+8h), 4 consecutive n
   const bool arow = m0 + am < P.M, bcol = n0 + bn + 3 < P.N;
   const float* Ap = P.A + (int64_t)(m0 + am) * P.lda + ak;
   const float* Bp = P.B + (int64_t)bk * P.ldb + n0 + bn;
-  float4 ra, rb;
+  float4 ra[H], rb[H];
   auto gload = [&](int k0) {
-    ra = make_float4(0.f, 0.f, 0.f, 0.f);
-    rb = ra;
-    if (arow) {
-      if (k0 + ak + 3 < P.K) ra = __ldg(reinterpret_cast<const float4*>(Ap + k0));
-      else {
-        float t[4];
-        for (int j = 0; j < 4; ++j) t[j] = (k0 + ak + j < P.K) ? __ldg(Ap + k0 + j) : 0.f;
-        ra = make_float4(t[0], t[1], t[2], t[3]);
+#pragma unroll
+    for (int h = 0; h < H; ++h) {
+      const int kh = k0 + 8 * h;
+      ra[h] = make_float4(0.f, 0.f, 0.f, 0.f);
+      rb[h] = ra[h];
+      if (arow) {
+        if (kh + ak + 3 < P.K) ra[h] = __ldg(reinterpret_cast<const float4*>(Ap + kh));
+        else {
+          float t[4];
+          for (int j = 0; j < 4; ++j) t[j] = (kh + ak + j < P.K) ? __ldg(Ap + kh + j) : 0.f;
+          ra[h] = make_float4(t[0], t[1], t[2], t[3]);
+        }
       }
-    }
-    if (k0 + bk < P.K) {
-      const float* b = Bp + (int64_t)k0 * P.ldb;
-      if (bcol) rb = __ldg(reinterpret_cast<const float4*>(b));
-      else {
-        float t[4];
-        for (int j = 0; j < 4; ++j) t[j] = (n0 + bn + j < P.N) ? __ldg(b + j) : 0.f;
-        rb = make_float4(t[0], t[1], t[2], t[3]);
+      if (kh + bk < P.K) {
+        const float* b = Bp + (int64_t)kh * P.ldb;
+        if (bcol) rb[h] = __ldg(reinterpret_cast<const float4*>(b));
+        else {
+          float t[4];
+          for (int j = 0; j < 4; ++j) t[j] = (n0 + bn + j < P.N) ? __ldg(b + j) : 0.f;
+          rb[h] = make_float4(t[0], t[1], t[2], t[3]);
+        }
       }
     }
   };
   auto sstore = [&](int buf) {
-    As[buf][ak + 0][am] = ra.x;
-    As[buf][ak + 1][am] = ra.y;
-    As[buf][ak + 2][am] = ra.z;
-    As[buf][ak + 3][am] = ra.w;
-    *reinterpret_cast<float4*>(&Bs[buf][bk][bn]) = rb;
+#pragma unroll
+    for (int h = 0; h < H; ++h) {
+      As[buf][8 * h + ak + 0][am] = ra[h].x;
+      As[buf][8 * h + ak + 1][am] = ra[h].y;
+      As[buf][8 * h + ak + 2][am] = ra[h].z;
+      As[buf][8 * h + ak + 3][am] = ra[h].w;
+      *reinterpret_cast<float4*>(&Bs[buf][8 * h + bk][bn]) = rb[h];
+    }
   };
   float acc[8][8];
 #pragma unroll
@@ -207,9 +216,9 @@ __global__ void __launch_bounds__(256, FP ? 1 : 2) t3_linear_kernel(const __grid
   sstore(0);
   __syncthreads();
   int buf = 0;
-  for (int k0 = 0; k0 < P.K; k0 += 8) {
-    const bool more = k0 + 8 < P.K;
-    if (more) gload(k0 + 8);
+  for (int k0 = 0; k0 < P.K; k0 += KB) {
+    const bool more = k0 + KB < P.K;
+    if (more) gload(k0 + KB);
     if (FP) {
       float4 fa[2][2], fb[2][2];
       fa[0][0] = *reinterpret_cast<const float4*>(&As[buf][0][ty * 4]);
@@ -217,9 +226,9 @@ __global__ void __launch_bounds__(256, FP ? 1 : 2) t3_linear_kernel(const __grid
       fb[0][0] = *reinterpret_cast<const float4*>(&Bs[buf][0][tx * 4]);
       fb[0][1] = *reinterpret_cast<const float4*>(&Bs[buf][0][64 + tx * 4]);
 #pragma unroll
-      for (int kk = 0; kk < 8; ++kk) {
+      for (int kk = 0; kk < KB; ++kk) {
         const int cur = kk & 1, nxt = cur ^ 1;
-        if (kk < 7) {
+        if (kk < KB - 1) {
           fa[nxt][0] = *reinterpret_cast<const float4*>(&As[buf][kk + 1][ty * 4]);
           fa[nxt][1] = *reinterpret_cast<const float4*>(&As[buf][kk + 1][64 + ty * 4]);
           fb[nxt][0] = *reinterpret_cast<const float4*>(&Bs[buf][kk + 1][tx * 4]);
@@ -236,7 +245,7 @@ __global__ void __launch_bounds__(256, FP ? 1 : 2) t3_linear_kernel(const __grid
       }
     } else {
 #pragma unroll
-    for (int kk = 0; kk < 8; ++kk) {
+    for (int kk = 0; kk < KB; ++kk) {
       const float4 a0 = *reinterpret_cast<const float4*>(&As[buf][kk][ty * 4]);
       const float4 a1 = *reinterpret_cast<const float4*>(&As[buf][kk][64 + ty * 4]);
       const float4 b0 = *reinterpret_cast<const float4*>(&Bs[buf][kk][tx * 4]);
@@ -402,9 +411,9 @@ mdh_status launch_t3(const Plan& p, const void* const* in, void* const* out, voi
     L.ldc = (int)p.auxi[3];
     dim3 grid((unsigned)((c.N + 127) / 128), (unsigned)((c.M + 127) / 128));
     if (grid.y > 65535) { set_error("T3: grid too large"); return MDH_ERR_UNSUPPORTED; }
-    // default: the fragment-pipelined one-CTA-per-SM variant (MatMul 4096³ fp32 3.05 ms,
-    // 60 % of FFMA, vs 3.80 ms for two 128-register CTAs per SM); tile knob stages=1 selects
-    // the latter
+    // default: the fragment-pipelined one-CTA-per-SM variant with 16-deep k-blocks (MatMul
+    // 4096³ fp32 2.94 ms, 63 % of FFMA; 3.05 ms with 8-deep k-blocks; 3.80 ms for two
+    // 128-register CTAs per SM); tile knob stages=1 selects the latter
     if (p.tiles.stages == 1) t3_linear_kernel<false><<<grid, 256, 0, st>>>(L);
     else t3_linear_kernel<true><<<grid, 256, 0, st>>>(L);
     return post_launch("t3_linear_kernel");
