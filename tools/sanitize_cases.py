@@ -30,6 +30,14 @@ def cases():
         "t4_split": (lambda: S.matmul(1280, 768, 512, "bf16"), "positive", "split=3"),
         "t4_ag": (lambda: S.mcc(4, 7, 7, 64, 3, 3, 16, "bf16"), "positive", None),
         "t4_split1": (lambda: S.matmul(2500, 2000, 512, "bf16", out_dtype="bf16"), "positive", "split=2"),
+        "t4_sk": (lambda: S.matmul(512, 512, 2048, "bf16"), "positive", "split=2"),
+        "t4_wide_sk": (lambda: S.matmul(512, 1024, 1024, "bf16"), "positive", "bn=512,split=2"),
+        "t4_wide": (lambda: S.matmul(700, 1000, 512, "bf16"), "positive", "bn=512,split=1"),
+        "t4_xfold": (lambda: S.matmul(100, 300, 2048, "bf16"), "positive", None),
+        "t4_im2col": (lambda: S.mcc(4, 7, 7, 512, 3, 3, 512, "bf16"), "positive", None),
+        "t4_cl4": (lambda: S.matmul(700, 1000, 512, "bf16"), "positive", "cluster=4"),
+        "t1_sweep": (lambda: S.jacobi3d_sweep(12, 10, 70), "positive", None),
+        "t6_colfold": (lambda: S.mbbs(300, 1000), "positive", None),
         "t5": (lambda: S.prl(300, 2000), "prl", None),
         "t6": (lambda: S.prefix_sum([3, 9000], 1), "positive", None),
         "combine": (lambda: S.dot(5000, "i32"), "virtual", None),
