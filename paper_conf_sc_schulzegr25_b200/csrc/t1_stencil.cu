@@ -137,13 +137,15 @@ __global__ void __launch_bounds__(128) t1_j3d7_kernel(const __grid_constant__ J7
       acc = fmaf(P.wzp, rp[j + 1], acc);
       o[j] = acc;
     }
+    // streaming (evict-first) stores: the output is never re-read, so it should not push
+    // the input rows that neighbouring CTAs still read (their y±1 rows) out of L2
     if (VEC_OUT == 1 && full) {
-      reinterpret_cast<float2*>(po)[0] = make_float2(o[0], o[1]);
-      reinterpret_cast<float2*>(po)[1] = make_float2(o[2], o[3]);
+      __stcs(reinterpret_cast<float2*>(po), make_float2(o[0], o[1]));
+      __stcs(reinterpret_cast<float2*>(po) + 1, make_float2(o[2], o[3]));
     } else if (VEC_OUT == 2 && full) {
-      po[0] = o[0];
-      *reinterpret_cast<float2*>(po + 1) = make_float2(o[1], o[2]);
-      po[3] = o[3];
+      __stcs(po, o[0]);
+      __stcs(reinterpret_cast<float2*>(po + 1), make_float2(o[1], o[2]));
+      __stcs(po + 3, o[3]);
     } else {
 #pragma unroll
       for (int j = 0; j < 4; ++j)
