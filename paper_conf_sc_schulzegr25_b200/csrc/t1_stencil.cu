@@ -92,42 +92,47 @@ struct J7Params {
   int64_t hbase;
 };
 
-template <bool VEC>
-__device__ __forceinline__ void row6(const float* p, bool full, int64_t rem, float r[6]) {
-  // r[k] = p[k], k = 0..5  (p = the x0-1 position); rem = number of valid positions
+// r[k] = p[k], k = 0..NX+1 (p = the x0-1 position, 16-byte aligned when VEC); rem = the
+// number of valid positions
+template <bool VEC, int NX>
+__device__ __forceinline__ void rowq(const float* p, bool full, int64_t rem, float* r) {
   if (VEC && full) {
-    const float4 a = __ldg(reinterpret_cast<const float4*>(p));
-    const float2 b = __ldg(reinterpret_cast<const float2*>(p + 4));
-    r[0] = a.x; r[1] = a.y; r[2] = a.z; r[3] = a.w; r[4] = b.x; r[5] = b.y;
+#pragma unroll
+    for (int q = 0; q < NX / 4; ++q) {
+      const float4 a = __ldg(reinterpret_cast<const float4*>(p) + q);
+      r[4 * q] = a.x; r[4 * q + 1] = a.y; r[4 * q + 2] = a.z; r[4 * q + 3] = a.w;
+    }
+    const float2 b = __ldg(reinterpret_cast<const float2*>(p + NX));
+    r[NX] = b.x; r[NX + 1] = b.y;
   } else {
 #pragma unroll
-    for (int k = 0; k < 6; ++k) r[k] = k < rem ? __ldg(p + k) : 0.f;
+    for (int k = 0; k < NX + 2; ++k) r[k] = k < rem ? __ldg(p + k) : 0.f;
   }
 }
-
-// VEC_OUT: 0 scalar stores; 1 two 8-byte stores (even output base); 2 odd output base
-// (e.g. the same-shape sweep of reading C-34, v[z+1,y+1,x+1]): scalar, 8-byte, scalar
-template <bool VEC_IN, int VEC_OUT>
+// VEC_OUT: 0 scalar stores; 1 8-byte stores (even output base); 2 odd output base
+// (e.g. the same-shape sweep of reading C-34, v[z+1,y+1,x+1]): scalar, 8-byte…, scalar.
+// NX: x outputs per thread (4, or 8 with tile knob vec=8)
+template <bool VEC_IN, int VEC_OUT, int NX>
 __global__ void __launch_bounds__(128) t1_j3d7_kernel(const __grid_constant__ J7Params P) {
-  const int x0 = (blockIdx.x * blockDim.x + threadIdx.x) * 4;
+  const int x0 = (blockIdx.x * blockDim.x + threadIdx.x) * NX;
   const int y = blockIdx.y * blockDim.y + threadIdx.y;
   if (x0 >= P.X || y >= P.Y) return;
   const int z0 = blockIdx.z * P.zchunk;
   const int z1 = min(P.Z, z0 + P.zchunk);
-  const bool full = x0 + 4 <= P.X;
+  const bool full = x0 + NX <= P.X;
   const int64_t rem = (int64_t)P.X + 1 - x0 + 1;     // valid positions x0-1 … X (centre-relative)
   const float* pc = P.u + P.bc - 1 + x0 + (int64_t)y * P.Ly + (int64_t)z0 * P.Lz;
   float* po = P.v + P.ob + x0 + (int64_t)y * P.oLy + (int64_t)z0 * P.oLz;
-  float rm[6], r0[6], rp[6], ym[6], yp[6];
-  row6<VEC_IN>(pc - P.Lz, full, rem, rm);
-  row6<VEC_IN>(pc, full, rem, r0);
+  float rm[NX + 2], r0[NX + 2], rp[NX + 2], ym[NX + 2], yp[NX + 2];
+  rowq<VEC_IN, NX>(pc - P.Lz, full, rem, rm);
+  rowq<VEC_IN, NX>(pc, full, rem, r0);
   for (int z = z0; z < z1; ++z) {
-    row6<VEC_IN>(pc + P.Lz, full, rem, rp);
-    row6<VEC_IN>(pc - P.Ly, full, rem, ym);
-    row6<VEC_IN>(pc + P.Ly, full, rem, yp);
-    float o[4];
+    rowq<VEC_IN, NX>(pc + P.Lz, full, rem, rp);
+    rowq<VEC_IN, NX>(pc - P.Ly, full, rem, ym);
+    rowq<VEC_IN, NX>(pc + P.Ly, full, rem, yp);
+    float o[NX];
 #pragma unroll
-    for (int j = 0; j < 4; ++j) {
+    for (int j = 0; j < NX; ++j) {
       float acc = P.wc * r0[j + 1];
       acc = fmaf(P.wxm, r0[j], acc);
       acc = fmaf(P.wxp, r0[j + 2], acc);
@@ -140,32 +145,33 @@ __global__ void __launch_bounds__(128) t1_j3d7_kernel(const __grid_constant__ J7
     // streaming (evict-first) stores: the output is never re-read, so it should not push
     // the input rows that neighbouring CTAs still read (their y±1 rows) out of L2
     if (VEC_OUT == 1 && full) {
-      __stcs(reinterpret_cast<float2*>(po), make_float2(o[0], o[1]));
-      __stcs(reinterpret_cast<float2*>(po) + 1, make_float2(o[2], o[3]));
+#pragma unroll
+      for (int j = 0; j < NX; j += 2) __stcs(reinterpret_cast<float2*>(po + j), make_float2(o[j], o[j + 1]));
     } else if (VEC_OUT == 2 && full) {
       __stcs(po, o[0]);
-      __stcs(reinterpret_cast<float2*>(po + 1), make_float2(o[1], o[2]));
-      __stcs(po + 3, o[3]);
+#pragma unroll
+      for (int j = 1; j + 1 < NX; j += 2) __stcs(reinterpret_cast<float2*>(po + j), make_float2(o[j], o[j + 1]));
+      __stcs(po + NX - 1, o[NX - 1]);
     } else {
 #pragma unroll
-      for (int j = 0; j < 4; ++j)
+      for (int j = 0; j < NX; ++j)
         if (x0 + j < P.X) po[j] = o[j];
     }
     float* ph = z == 0 ? P.hlo : (z == P.Z - 1 ? P.hhi : nullptr);
     if (ph) {                      // this plane is also a neighbour's halo plane
       ph += P.hbase + x0 + (int64_t)y * P.oLy;
 #pragma unroll
-      for (int j = 0; j < 4; ++j)
+      for (int j = 0; j < NX; ++j)
         if (x0 + j < P.X) ph[j] = o[j];
     }
     if (P.hlo && P.hhi && P.Z == 1) {   // a one-plane slab feeds both neighbours
       float* q = P.hhi + P.hbase + x0 + (int64_t)y * P.oLy;
 #pragma unroll
-      for (int j = 0; j < 4; ++j)
+      for (int j = 0; j < NX; ++j)
         if (x0 + j < P.X) q[j] = o[j];
     }
 #pragma unroll
-    for (int k = 0; k < 6; ++k) { rm[k] = r0[k]; r0[k] = rp[k]; }
+    for (int k = 0; k < NX + 2; ++k) { rm[k] = r0[k]; r0[k] = rp[k]; }
     pc += P.Lz;
     po += P.oLz;
   }
@@ -438,14 +444,23 @@ static mdh_status launch_j3d7(const Plan& p, const void* const* in, void* const*
   // (32 / 64 / 128).  Measured on 512³ (zchunk 8): 32 → 206.8 µs, 64 → 209.0, 128 → 219.2 —
   // the y-halo rows of a narrow, tall block are L1 hits; longer row segments do not pay
   const int bx = (p.tiles.per_thread == 64 || p.tiles.per_thread == 128) ? p.tiles.per_thread : 32;
+  // x outputs per thread: 4, or 8 with tile knob vec=8 (measured 292.9 vs 208.8 µs on 512³:
+  // half the threads per plane row leave too few loads in flight)
+  const int nx = p.tiles.vec == 8 ? 8 : 4;
   dim3 block(bx, 128 / bx);
-  dim3 grid((unsigned)((P.X + 4 * bx - 1) / (4 * bx)), (unsigned)((P.Y + block.y - 1) / block.y),
+  dim3 grid((unsigned)((P.X + nx * bx - 1) / (nx * bx)), (unsigned)((P.Y + block.y - 1) / block.y),
             (unsigned)((P.Z + zc - 1) / zc));
-  if (vin && vout) t1_j3d7_kernel<true, 1><<<grid, block, 0, st>>>(P);
-  else if (vin && vodd) t1_j3d7_kernel<true, 2><<<grid, block, 0, st>>>(P);
-  else if (vin) t1_j3d7_kernel<true, 0><<<grid, block, 0, st>>>(P);
-  else if (vout) t1_j3d7_kernel<false, 1><<<grid, block, 0, st>>>(P);
-  else t1_j3d7_kernel<false, 0><<<grid, block, 0, st>>>(P);
+#define J7(VI, VO)                                                        \
+  do {                                                                    \
+    if (nx == 8) t1_j3d7_kernel<VI, VO, 8><<<grid, block, 0, st>>>(P);   \
+    else t1_j3d7_kernel<VI, VO, 4><<<grid, block, 0, st>>>(P);           \
+  } while (0)
+  if (vin && vout) J7(true, 1);
+  else if (vin && vodd) J7(true, 2);
+  else if (vin) J7(true, 0);
+  else if (vout) J7(false, 1);
+  else J7(false, 0);
+#undef J7
   return post_launch("t1_j3d7_kernel");
 }
 
