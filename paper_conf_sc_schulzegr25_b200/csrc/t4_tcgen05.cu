@@ -1480,6 +1480,7 @@ struct T4State {
   int cg = 1;      // 1: one SM per 128×256 tile; 2: SM pair per 256×256 tile
   int cl = 2;      // 2-SM kernel: CTAs per cluster (4: two pairs share B by multicast)
   int nw = 256;    // 2-SM kernel: N extent of a pair tile (512: two MMAs per k-step)
+  bool sk_ok = false;   // 2-SM kernel: stream-K workspace reserved
   bool ag = false; // A staged by the kernel's gather warps (no A tensor map, no pre-pass)
   bool ic = false;  // A through a TMA im2col map
   uint64_t ic_dims[4];
@@ -1746,10 +1747,15 @@ mdh_status prepare_t4(Plan* p) {
       P.tiles_n = (int)((c.N + 511) / 512);
       P.num_tiles = P.tiles_m * P.tiles_n;
     }
-    // room for the stream-K partial tiles and flags (decided at launch from the SM count)
-    ws = (ws + 255) / 256 * 256;
-    s->tail_off = ws;
-    ws += (size_t)t4::SK_MAX_PAIRS * (s->nw / 256) * 65536 * sizeof(float) + 16 * t4::SK_MAX_PAIRS * sizeof(unsigned) + 256;
+    // room for the stream-K partial tiles and flags, only when stream-K can be chosen at
+    // launch (forced, or the auto rule: one partial wave of deep tiles — fewer tiles than
+    // pairs, and the launch never has more pairs than SMs/2)
+    s->sk_ok = p->tiles.split >= 2 || (p->tiles.split == 0 && P.num_tiles < plan_sms(p) / 2 && P.num_kb >= 64);
+    if (s->sk_ok) {
+      ws = (ws + 255) / 256 * 256;
+      s->tail_off = ws;
+      ws += (size_t)t4::SK_MAX_PAIRS * (s->nw / 256) * 65536 * sizeof(float) + 16 * t4::SK_MAX_PAIRS * sizeof(unsigned) + 256;
+    }
   } else {
     // 1-SM split-K tail: the T mod C tiles of the last, partial wave split along K over
     // the idle SMs (S units each) — tile knob split=S, or automatically when the partial
@@ -2103,7 +2109,7 @@ mdh_status launch_t4(const Plan& p, const void* const* in, void* const* out, voi
     // 32.7 vs 24.6 µs; tools/sweep_tiles.py).  Tile knob split=1 never, split≥2 whenever
     // the last wave is partial.
     const bool sk_auto = T < C && P.num_kb >= 64;
-    if (T % C != 0 && (p.tiles.split >= 2 || (p.tiles.split == 0 && sk_auto))) {
+    if (s->sk_ok && T % C != 0 && (p.tiles.split >= 2 || (p.tiles.split == 0 && sk_auto))) {
       // every complete wave runs whole tiles (their epilogues overlap later MMAs); only the
       // partial last wave is spread over all pairs, so few outputs are written at the end
       const int nfull = R * C;
