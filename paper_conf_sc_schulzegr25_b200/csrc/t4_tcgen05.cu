@@ -78,7 +78,9 @@ struct Params {
   const uint16_t* Ag;
   const int64_t* aM;
   const int64_t* aK;                // offA_K table (every 8th entry is a chunk start)
-  int nkc;                          // K / 8 chunk offsets staged in shared memory
+  int nkc;                          // K / 8 (K / 4 with ag4) chunk offsets staged in shared memory
+  int ag4;                          // gather in 8-byte runs of 4 (K offsets contiguous in runs of 4)
+  int run4;                         // EPI 2 with runs of 4 (fp32: 16-byte stores) instead of 8
   int ag_lag;                       // k-blocks between issuing a stage and publishing it (1..3)
   // bulk-run epilogue (EPI 3): N-tile = 2 output runs of bn/2 contiguous elements
   int bn;                           // N-tile width (EPI 3; else BN)
@@ -492,8 +494,55 @@ __global__ void __launch_bounds__(AG ? THREADS + AG_THREADS : THREADS, 1)
     // materialised im2col / permuted copy.  Thread → K chunk (gt & 7) of rows gt/8 + 16 i.
     // A stage is published AG_LAG k-blocks later: wait_group, proxy fence, arrive.
     const int gt = threadIdx.x - THREADS;
-    for (int i = gt; i < P.nkc; i += AG_THREADS) s_koff[i] = __ldg(P.aK + 8 * (int64_t)i);
+    const int run = P.ag4 ? 4 : 8;
+    for (int i = gt; i < P.nkc; i += AG_THREADS) s_koff[i] = __ldg(P.aK + run * (int64_t)i);
     named_sync(2, AG_THREADS);
+    if (P.ag4) {
+      // 8-byte variant (K offsets contiguous only in runs of 4, e.g. MCC_Caps' l): thread →
+      // half-chunk (gt & 15) of rows gt/16 + 8 i; half h of 16-B chunk c of row r at
+      // ((c ^ (r & 7)) * 16 + 8 h)
+      const int hc = gt & 15, rb4 = gt >> 4;
+      int stage = 0;
+      uint32_t phase = 0;
+      int g = 0;
+      for (int u = u_first(P); u < u_last(P); u += u_step(P)) {
+        int mb, nb, kb0, kb1, slot;
+        u_decode(P, u, &mb, &nb, &kb0, &kb1, &slot);
+        const int64_t m0 = (int64_t)mb * BM;
+        int64_t ro[16];
+#pragma unroll
+        for (int i = 0; i < 16; ++i) {
+          const int64_t m = m0 + rb4 + 8 * i;
+          ro[i] = m < P.M ? __ldg(P.aM + m) : -1;
+        }
+        for (int kb = kb0; kb < kb1; ++kb, ++g) {
+          mbar_wait(empty0 + 8 * stage, phase ^ 1);
+          const uint32_t base = smem_u32(sA + stage * A_BYTES);
+          const int kc = krotate(P, kb, kb0, kb1, (int)mb) * (BK / 4) + hc;
+          const int64_t ko = kc < P.nkc ? s_koff[kc] : -1;
+#pragma unroll
+          for (int i = 0; i < 16; ++i) {
+            const int r = rb4 + 8 * i;
+            const uint32_t dst = base + r * 128 + (((hc >> 1) ^ (r & 7)) << 4) + ((hc & 1) << 3);
+            if (ro[i] >= 0 && ko >= 0)
+              asm volatile("cp.async.ca.shared.global [%0], [%1], 8;" ::"r"(dst), "l"(P.Ag + ro[i] + ko) : "memory");
+            else asm volatile("st.shared.v2.u32 [%0], {%1, %1};" ::"r"(dst), "r"(0) : "memory");
+          }
+          cp_async_commit();
+          if (g >= P.ag_lag) {
+            if (P.ag_lag == 1) cp_async_wait<1>();
+            else if (P.ag_lag == 2) cp_async_wait<2>();
+            else cp_async_wait<3>();
+            fence_proxy_async();
+            mbar_arrive(full0 + 8 * ((g - P.ag_lag) % NST));
+          }
+          if (++stage == NST) { stage = 0; phase ^= 1; }
+        }
+      }
+      cp_async_wait<0>();
+      fence_proxy_async();
+      for (int j = g - P.ag_lag < 0 ? 0 : g - P.ag_lag; j < g; ++j) mbar_arrive(full0 + 8 * (j % NST));
+    } else {
     const int ch = gt & 7, rb = gt >> 3;
     int stage = 0;
     uint32_t phase = 0;
@@ -534,6 +583,7 @@ __global__ void __launch_bounds__(AG ? THREADS + AG_THREADS : THREADS, 1)
     cp_async_wait<0>();
     fence_proxy_async();
     for (int j = g - P.ag_lag < 0 ? 0 : g - P.ag_lag; j < g; ++j) mbar_arrive(full0 + 8 * (j % NST));
+    }
   } else if (EPI == 3) {
     // ===== bulk-run epilogue: the output is contiguous along n in runs of L = bn/2 and a
     // warp owns 32 accumulator rows × one run.  TMEM → registers → this warp's staging
@@ -722,7 +772,19 @@ __global__ void __launch_bounds__(AG ? THREADS + AG_THREADS : THREADS, 1)
           // run-8 scatter: the output is contiguous along n in aligned runs of 8 (the plan
           // checked cN and the alignment), so each thread stores its row's 32 columns as
           // four 32-byte vectors (STG.256; 16 B for bf16) at crow + cN[run start]
-          if (mok) {
+          if (mok && P.run4 && !OUT_BF16) {
+            // run-4: eight 16-byte vectors at crow + cN[run start]
+#pragma unroll
+            for (int j = 0; j < 8; ++j) {
+              if (nb + 4 * j < P.N) {
+                const int64_t o = crow + s_cn[half * (BN / 2) + c * 32 + 4 * j];
+                const uint32_t* v = r + 4 * j;
+                asm volatile("st.global.cs.v4.b32 [%0], {%1, %2, %3, %4};" ::"l"(P.C + o), "r"(v[0]), "r"(v[1]), "r"(v[2]),
+                             "r"(v[3])
+                             : "memory");
+              }
+            }
+          } else if (mok) {
 #pragma unroll
             for (int j = 0; j < 4; ++j) {
               if (nb + 8 * j < P.N) {
@@ -1655,6 +1717,23 @@ mdh_status prepare_t4(Plan* p) {
     for (size_t i = 0; i < tm.size() && a_gather; ++i)
       if (tm[i] % 8) a_gather = false;
   }
+  // 8-byte gather: K offsets contiguous only in aligned runs of 4 (MCC_Caps' capsule dim l)
+  bool a_gather4 = false;
+  if (!a_2d && !a_box && !a_ic && !a_gather && (p->tiles.implicit == 0 || p->tiles.implicit == 2) && c.K % 4 == 0 &&
+      c.K / 4 <= t4::KOFF_MAX) {
+    std::vector<int64_t> tk = t4::table(*p, c.kd, c.nk, p->in[c.a_buf].acc[0]);
+    std::vector<int64_t> tm = t4::table(*p, c.md, c.nm, p->in[c.a_buf].acc[0]);
+    const int64_t base = p->in[c.a_buf].acc[0].base;
+    a_gather4 = true;
+    for (size_t i = 0; i < tk.size() && a_gather4; i += 4) {
+      if ((tk[i] + base) % 4) a_gather4 = false;
+      for (int j = 1; j < 4 && a_gather4; ++j)
+        if (tk[i + j] != tk[i] + j) a_gather4 = false;
+    }
+    for (size_t i = 0; i < tm.size() && a_gather4; ++i)
+      if (tm[i] % 4) a_gather4 = false;
+    if (a_gather4) a_gather = true;
+  }
   if (a_box || a_gather || a_ic) {
     s->a = t4::Layout2D();
     s->a.ok = true;
@@ -1716,12 +1795,28 @@ mdh_status prepare_t4(Plan* p) {
       if (cm[i] % 8) run8 = false;
     if (run8) s->epi = 2;
   }
+  // run-4 variant (fp32 output; MCC_Caps: res[…, k, i, j] with j the 4-run between k and i)
+  if (!P.c_rowmajor && s->epi == 1 && c.N % 4 == 0 && p->out[0].dtype == MDH_F32) {
+    bool run4 = true;
+    for (size_t i = 0; i < cn.size() && run4; i += 4) {
+      if ((P.cbase + cn[i]) % 4) run4 = false;
+      for (int j = 1; j < 4 && run4; ++j)
+        if (cn[i + j] != cn[i] + j) run4 = false;
+    }
+    for (size_t i = 0; i < cm.size() && run4; ++i)
+      if (cm[i] % 4) run4 = false;
+    if (run4) {
+      s->epi = 2;
+      P.run4 = 1;
+    }
+  }
   // 2-SM pairs (cta_group::2, 256×256 tiles) for large row-major outputs (measured 1290 vs
   // 1170 TFLOP/s on MatMul 4096³); tile knob cluster=1 forces the 1-SM kernel
   // (the in-kernel A gather is a 1-SM kernel: a 2-SM version, whose peer CTA must publish
   // its gathered half at cluster scope, measured 86-208 µs vs 83 µs on MCC conv5_1)
   s->ag = a_gather;
-  P.nkc = (int)(c.K / 8);
+  P.ag4 = a_gather4 ? 1 : 0;
+  P.nkc = (int)(c.K / (a_gather4 ? 4 : 8));
   s->cg = (!a_gather && P.c_rowmajor && !P.out_bf16 && c.M >= 256 && c.N >= 256 && p->tiles.cluster != 1) ? 2 : 1;
   if (s->cg == 2) {
     P.tiles_m = (int)((c.M + 255) / 256);
@@ -2156,7 +2251,7 @@ mdh_status launch_t4(const Plan& p, const void* const* in, void* const* out, voi
     P.tail_cnt = (unsigned*)((char*)ws + s->tail_off + (size_t)s->tail_parts * t4::BM * t4::BN * sizeof(float));
   }
   // EPI 2 needs a 32-byte (fp32) / 16-byte (bf16) aligned output base
-  const bool epi2 = s->epi == 2 && (uintptr_t)P.C % (P.out_bf16 ? 16 : 32) == 0;
+  const bool epi2 = s->epi == 2 && (uintptr_t)P.C % (P.out_bf16 || P.run4 ? 16 : 32) == 0;
   if (s->ag) {
     P.ag_lag = 2;   // measured on MCC conv5_1: lag 1 / 2 / 3 → 89 / 83 / 130 µs
     constexpr int TG = t4::THREADS + t4::AG_THREADS;
