@@ -129,6 +129,13 @@ typedef struct {
 
 #define MDH_PLAN_VIRTUAL_SHARD 0x1u  /* plan rank r of world_size on one GPU, no comm */
 #define MDH_PLAN_NO_COLLECTIVE 0x2u  /* pw shard: leave the partial result local       */
+#define MDH_PLAN_FLOAT_ALLREDUCE 0x4u /* pw(add) shard of a float output: ncclAllReduce
+                                        (NVLS in-switch reduction where NCCL selects it)
+                                        instead of allgather + ordered combine — faster
+                                        for large outputs (split-K MatMul / MCC across
+                                        GPUs), but the summation order
+                                        is NCCL's: reproducible only for a fixed NCCL
+                                        algorithm and topology                          */
 
 typedef struct {
   int32_t device;        /* CUDA device ordinal the plan executes on                   */

@@ -141,7 +141,10 @@ static mdh_status execute_sharded(const mdh::Plan& p, const void* const* in, voi
   bool exact_any_order = p.n_out == 1 && p.f != MDH_F_PRL_COMPARE &&
                          (p.redop == MDH_PW_MAX || p.redop == MDH_PW_MIN ||
                           (p.redop == MDH_PW_ADD && !is_float(p.out[0].dtype)));
-  if (exact_any_order) {
+  // opt-in: float sums through NCCL's reduction (order chosen by NCCL)
+  const bool float_allreduce = (p.flags & MDH_PLAN_FLOAT_ALLREDUCE) && p.n_out == 1 && p.f != MDH_F_PRL_COMPARE &&
+                               p.redop == MDH_PW_ADD && (p.out[0].dtype == MDH_F32 || p.out[0].dtype == MDH_F64);
+  if (exact_any_order || float_allreduce) {
     return comm_allreduce(p.comm, lout[0], out[0], (size_t)p.out[0].elems, p.out[0].dtype, p.redop, st);
   }
   MDH_TRY(comm_allgather(p.comm, local, gathered, per, st));

@@ -30,6 +30,7 @@ STATUS = {0: "OK", 1: "INVALID_ARG", 2: "INVALID_SPEC", 3: "UNSUPPORTED", 4: "OU
           5: "CUDA", 6: "NCCL", 7: "INTERNAL"}
 VIRTUAL_SHARD = 0x1
 NO_COLLECTIVE = 0x2
+FLOAT_ALLREDUCE = 0x4                # include/mdh.h MDH_PLAN_FLOAT_ALLREDUCE
 
 
 class IndexFn(ctypes.Structure):
