@@ -102,3 +102,51 @@ def test_sweeps_rejects_bad_plans():
     h.rank, h.world = 1, 2                           # no transport given
     with pytest.raises(MdhError):
         q.stencil_sweeps(u, u.clone(), 1, halo=h)
+
+
+def _box3_sweep(Y, X):
+    """A 2-D 3×3 same-shape stencil sweep (v[i+1, j+1] = Σ w_rs·u[i+r, j+s], boundary ring
+    kept) — runs on the box-window kernel, so the peer transport falls back to copies."""
+    d = ["i", "j"]
+    accs = [[f"i+{r}", f"j+{c}"] for r in range(3) for c in range(3)]
+    wts = [0.05, 0.1, 0.05, 0.1, 0.3, 0.1, 0.05, 0.1, 0.05]
+    return S.make_spec("box3_sweep", d, [Y - 2, X - 2], ["CC", "CC"], "STENCIL",
+                       [S.buffer("u", "f32", accs, d, shape=[Y, X])],
+                       [S.buffer("v", "f32", [["i+1", "j+1"]], d, shape=[Y, X])], fparams=wts)
+
+
+@pytest.mark.parametrize("world", [1, 3])
+def test_sweeps_box2d_copy_transport(world):
+    """Non-7-point stencil: the sweep kernel cannot store halos itself, so after each sweep
+    the boundary rows are copied into the neighbours' halo rows (device-to-device)."""
+    import torch
+    from paper_conf_sc_schulzegr25_b200 import Halo, Plan
+    Y, X, T = 29, 68, 3
+    u0 = _field(1, Y, X, 3430)[0]
+    sp = _box3_sweep(Y, X)
+    ref = oracle.stencil_sweeps(sp, u0, T)
+    slabs = S.z_slabs(Y, world)
+    bufs, plans = [], []
+    for lo, hi in slabs:
+        b0 = torch.from_numpy(np.ascontiguousarray(u0[lo - 1:hi + 1])).cuda()
+        bufs.append([b0, b0.clone()])
+        plans.append(Plan(_box3_sweep(hi - lo + 2, X)))
+    row = X * 4
+    for t in range(T):
+        s, d = t & 1, (t & 1) ^ 1
+        for r, (lo, hi) in enumerate(slabs):
+            h = Halo()
+            h.rank, h.world = r, world
+            if r > 0:
+                nzl = slabs[r - 1][1] - slabs[r - 1][0] + 2
+                for k, i in enumerate((s, d)):
+                    h.peer_lo[k] = bufs[r - 1][i].data_ptr() + (nzl - 1) * row
+            if r < world - 1:
+                for k, i in enumerate((s, d)):
+                    h.peer_hi[k] = bufs[r + 1][i].data_ptr()
+            plans[r].stencil_sweeps(bufs[r][s], bufs[r][d], 1, halo=h if world > 1 else None)
+    torch.cuda.synchronize()
+    for r, (lo, hi) in enumerate(slabs):
+        owned = bufs[r][T & 1].cpu().numpy()[1:hi - lo + 1].astype(np.float64)
+        assert np.max(np.abs(owned - ref[lo:hi])) <= 1e-5 * max(1.0, np.abs(ref).max())
+
