@@ -72,6 +72,7 @@ struct Tiles {
                                       // GEMM), 2 in-kernel cp.async gather, 3 gather pre-pass
   int epi = 0;                        // T4 scatter epilogue: 0 auto, 1 never the bulk-run (EPI 3) kernel
   int krot = 0;                       // T4 k-block rotation per tile (1 = on)
+  int l2pf = 0;                       // T1 7-point row loads: L2 prefetch hint 0 none, 1 128 B, 2 256 B
   std::string source = "default";
 };
 

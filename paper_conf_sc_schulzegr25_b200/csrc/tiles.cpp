@@ -146,6 +146,7 @@ void apply(Tiles* t, const std::string& k, double v) {
   else if (k == "implicit") t->implicit = iv;
   else if (k == "epi") t->epi = iv;
   else if (k == "krot") t->krot = iv;
+  else if (k == "l2pf") t->l2pf = iv;
 }
 
 std::string read_file(const char* path) {
