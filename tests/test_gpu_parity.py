@@ -110,6 +110,21 @@ def test_jacobi3d_full_size_sampled_and_closed_forms():
     assert np.abs(got[0].astype(np.float64) - g["constant_field_2_0"]).max() <= 1e-4 * 2.0 * 2.0 * 1.67
 
 
+@pytest.mark.parametrize("zyx", [(5, 7, 9), (66, 130, 258)])
+def test_jacobi3d_l2_prefetch_hint_variants(zyx):
+    """Tile knob l2pf (L2 prefetch-size hint on the 7-point row loads): a cache hint only, so
+    every setting is bit-identical to the others and within 1e-4 of the oracle."""
+    spec = S.jacobi3d(*zyx)
+    x = G.jacobi3d_inputs(*zyx)
+    outs = []
+    for pf in (0, 1, 2):
+        got, p = run_gpu(spec, x, force_tile=f"zchunk=8,l2pf={pf}")
+        assert p.template == "T1_stencil"
+        outs.append(got[0])
+    assert outs[0].tobytes() == outs[1].tobytes() == outs[2].tobytes()
+    assert_close_full(spec, x, [outs[2]], 1e-4, kind="scale")
+
+
 @pytest.mark.parametrize("IJ", [(1, 1), (3, 5), (17, 33), (224, 224), (129, 1030)])
 def test_gaussian2d(IJ):
     """Gaussian_2D 5×5 (reading C-31; Fig 3) on the 2-D box-window T1 kernel:
