@@ -775,7 +775,15 @@ __global__ void __launch_bounds__(T6T_THREADS, 1) t6_stream_scan_kernel(const __
     __syncthreads();
     const int k0 = tid * K, k1 = min(len, k0 + K);
     V ts = (V)0;
-    for (int k = k0; k < k1; ++k) ts = Arith<V>::add(ts, sb[k]);
+    if (k1 - k0 == K) {            // whole run: all K shared-memory loads issued before the adds
+      V v[K];
+#pragma unroll
+      for (int q = 0; q < K; ++q) v[q] = sb[k0 + q];
+#pragma unroll
+      for (int q = 0; q < K; ++q) ts = Arith<V>::add(ts, v[q]);
+    } else {
+      for (int k = k0; k < k1; ++k) ts = Arith<V>::add(ts, sb[k]);
+    }
     V incl = ts;
 #pragma unroll
     for (int o = 1; o < 32; o <<= 1) {
@@ -821,9 +829,20 @@ __global__ void __launch_bounds__(T6T_THREADS, 1) t6_stream_scan_kernel(const __
     const V prev = __shfl_up_sync(0xffffffffu, incl_cur, 1);
     V r = lane == 0 ? base : Arith<V>::add(base, prev);
     const int k0 = tid * K, k1 = min(len, k0 + K);
-    for (int k = k0; k < k1; ++k) {
-      r = Arith<V>::add(r, sb[k]);
-      sb[k] = r;
+    if (k1 - k0 == K) {            // whole run: loads first, then the sequential scan and stores
+      V v[K];
+#pragma unroll
+      for (int q = 0; q < K; ++q) v[q] = sb[k0 + q];
+#pragma unroll
+      for (int q = 0; q < K; ++q) {
+        r = Arith<V>::add(r, v[q]);
+        sb[k0 + q] = r;
+      }
+    } else {
+      for (int k = k0; k < k1; ++k) {
+        r = Arith<V>::add(r, sb[k]);
+        sb[k] = r;
+      }
     }
     asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
     __syncthreads();
