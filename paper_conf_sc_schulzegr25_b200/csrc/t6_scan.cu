@@ -147,6 +147,9 @@ __global__ void __launch_bounds__(1024) t6_fold_kernel(const __grid_constant__ T
 // inside a sub-range, sub-ranges (threadIdx.y, then blockIdx.y) ascending — fixed, so the
 // result is deterministic.
 __global__ void __launch_bounds__(256) t6_colfold_kernel(const __grid_constant__ T6Params P) {
+  // the row scan that follows is launched with programmatic stream serialization: let it
+  // be scheduled now (it waits in griddepcontrol.wait until this grid's writes are visible)
+  asm volatile("griddepcontrol.launch_dependents;" ::: "memory");
   __shared__ float4 part[8][32];
   __shared__ int last;
   const int64_t T = P.T;
@@ -271,6 +274,60 @@ __global__ void __launch_bounds__(1024) t6_rowscan_kernel(const __grid_constant_
   for (int64_t k = a0; k < a1; ++k) { run = Arith<V>::add(run, zs[k]); zs[k] = run; }
   __syncthreads();
   for (int64_t k = tid; k < T; k += 1024) store_as<V>(P.out, P.odt, t6_out_offset(P, c, k), zs[k]);
+}
+
+// The same scan for fp32 rows of T = 1024·4·nv elements (nv ≤ 8) and a contiguous, 16-byte
+// aligned fp32 output row: each thread's segment of T/1024 consecutive elements is held in
+// registers (float4 loads from the fold result, float4 stores to out) — no shared-memory
+// staging — with exactly the association of t6_rowscan_kernel (bit-identical results).
+// Launched as a programmatic dependent of the column fold: griddepcontrol.wait returns once
+// the fold grid has completed and its writes are visible.
+__global__ void __launch_bounds__(1024) t6_rowscan4_kernel(const __grid_constant__ T6Params P) {
+  asm volatile("griddepcontrol.wait;" ::: "memory");
+  __shared__ float wtot[32];
+  const int64_t c = blockIdx.x, T = P.T;
+  const int tid = threadIdx.x, lane = tid & 31, wid = tid >> 5;
+  const int nv = (int)(T / 4096);
+  const float4* zr = reinterpret_cast<const float4*>((const float*)P.z + c * T) + (int64_t)tid * nv;
+  float4 v[8];
+#pragma unroll
+  for (int q = 0; q < 8; ++q)
+    if (q < nv) v[q] = __ldcg(zr + q);
+  float sum = 0.f;
+#pragma unroll
+  for (int q = 0; q < 8; ++q)
+    if (q < nv) { sum += v[q].x; sum += v[q].y; sum += v[q].z; sum += v[q].w; }
+  float incl = sum;
+#pragma unroll
+  for (int o = 1; o < 32; o <<= 1) {
+    const float y = __shfl_up_sync(0xffffffffu, incl, o);
+    if (lane >= o) incl = y + incl;
+  }
+  float excl = __shfl_up_sync(0xffffffffu, incl, 1);
+  if (lane == 0) excl = 0.f;
+  if (lane == 31) wtot[wid] = incl;
+  __syncthreads();
+  if (wid == 0) {
+    float w = wtot[lane];
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+      const float y = __shfl_up_sync(0xffffffffu, w, o);
+      if (lane >= o) w = y + w;
+    }
+    wtot[lane] = w;
+  }
+  __syncthreads();
+  float run = wid > 0 ? wtot[wid - 1] + excl : excl;
+  float4* orow = reinterpret_cast<float4*>((float*)P.out + t6_out_offset(P, c, 0)) + (int64_t)tid * nv;
+#pragma unroll
+  for (int q = 0; q < 8; ++q)
+    if (q < nv) {
+      run += v[q].x; v[q].x = run;
+      run += v[q].y; v[q].y = run;
+      run += v[q].z; v[q].z = run;
+      run += v[q].w; v[q].w = run;
+      orow[q] = v[q];
+    }
 }
 
 // block inclusive scan of one chunk; writes either the final output (single chunk) or the
@@ -970,6 +1027,14 @@ static mdh_status launch_stream(T6Params& P, cudaStream_t st) {
   return post_launch("t6_stream_scan_kernel");
 }
 
+// every output row starts on a 16-byte boundary (float4 stores in t6_rowscan4_kernel)
+static bool row_out_aligned4(const T6Params& P) {
+  if (((uintptr_t)P.out & 15) != 0 || ((uintptr_t)P.z & 15) != 0 || P.obase % 4 != 0) return false;
+  for (int q = 0; q < P.nrowd; ++q)
+    if (P.orowL[q] % 4 != 0) return false;
+  return true;
+}
+
 template <class V>
 static mdh_status launch_typed(const T6Params& P, cudaStream_t st) {
   const int64_t total = P.Nc * P.T;
@@ -989,6 +1054,23 @@ static mdh_status launch_typed(const T6Params& P, cudaStream_t st) {
       t6_fold_kernel<V><<<gf, dim3(32, Y), 0, st>>>(P);
       MDH_TRY(post_launch("t6_fold_kernel"));
     }
+  }
+  if (std::is_same<V, float>::value && !P.direct && P.colS > 0 && P.odt == MDH_F32 && P.oLt == 1 &&
+      P.T % 4096 == 0 && P.T <= 8 * 4096 && P.Nc <= INT32_MAX && row_out_aligned4(P)) {
+    // fp32 rows after the column fold: register row scan, launched as a programmatic
+    // dependent of the fold (its launch and prologue overlap the fold's tail)
+    cudaLaunchConfig_t cfg = {};
+    cfg.gridDim = dim3((unsigned)P.Nc);
+    cfg.blockDim = dim3(1024);
+    cfg.dynamicSmemBytes = 0;
+    cfg.stream = st;
+    cudaLaunchAttribute attr[1];
+    attr[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+    attr[0].val.programmaticStreamSerializationAllowed = 1;
+    cfg.attrs = attr;
+    cfg.numAttrs = 1;
+    MDH_CUDA(cudaLaunchKernelEx(&cfg, t6_rowscan4_kernel, P));
+    return post_launch("t6_rowscan4_kernel");
   }
   if (!P.direct && P.T * (int64_t)sizeof(V) <= T6_ROW_SMEM && P.Nc <= INT32_MAX) {
     // short rows: one single-block scan per row instead of chunk scan + totals + fix-up

@@ -98,11 +98,14 @@ def test_gpu_single_pass_scan(shape, dt, tile):
 
 
 @gpu
-@pytest.mark.parametrize("IJ", [(64, 37), (1000, 5000), (4096, 8192), (8192, 8192), (300, 1000), (40, 64)])
+@pytest.mark.parametrize("IJ", [(64, 37), (1000, 5000), (4096, 8192), (8192, 8192), (300, 1000), (40, 64),
+                                (64, 4096), (16, 32768), (8, 12288)])
 def test_gpu_mbbs(IJ):
     """MBBS on T6; shapes with J % 4 == 0 take the column-fold K1 (16-byte column loads,
     the row range split over blocks, ordered ticket fold; ragged last column group for
-    J = 1000).  Run twice on one plan: tickets back at rest, results bit-identical."""
+    J = 1000); J = 4096·nv (nv = 1, 2, 3, 8) then take the register row scan launched as a
+    programmatic dependent of the fold.  Run twice on one plan: tickets back at rest,
+    results bit-identical."""
     from gpu_util import assert_close_full, run_gpu
     spec = S.mbbs(*IJ)
     x = G.gen_inputs(spec, 6200, "positive")
