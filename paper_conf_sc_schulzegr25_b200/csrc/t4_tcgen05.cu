@@ -338,6 +338,9 @@ __global__ void __launch_bounds__(AG ? THREADS + AG_THREADS : THREADS, 1)
                 const __grid_constant__ Params P) {
   extern __shared__ __align__(1024) uint8_t smem_raw[];
   __shared__ int64_t s_cn[BN];      // column offsets of the current N-tile (scatter epilogue)
+  // split-K over the idle SMs: the fold (t4_xfold_kernel, a programmatic dependent) may be
+  // scheduled now; it waits in griddepcontrol.wait for this grid's partials
+  if (P.xfold) asm volatile("griddepcontrol.launch_dependents;" ::: "memory");
   // ring: NST stages of A (16 KB) and B (bn·128 B); EPI 3 keeps 2 stages to leave room for
   // the epilogue's staging buffers (K is short where it is used: CCSD(T) K = 72)
   constexpr int NST = EPI == 3 ? 2 : STAGES;
@@ -1326,6 +1329,7 @@ __global__ void __cluster_dims__(CL, 1, 1) __launch_bounds__(THREADS, 1)
 // fp32 partial tiles [128][256]; fold them in split order (deterministic) across the whole
 // GPU and write through out_view (row-major or the offset tables; fp32 or bf16).
 __global__ void __launch_bounds__(256) t4_xfold_kernel(const __grid_constant__ Params P) {
+  asm volatile("griddepcontrol.wait;" ::: "memory");   // the GEMM grid's partials are visible
   constexpr int64_t PT = (int64_t)BM * BN;
   const int64_t per_tile = PT / 4;
   const int64_t total = (int64_t)(P.nunits / P.ssplit) * per_tile;
@@ -2045,7 +2049,17 @@ static mdh_status launch_xfold(const t4::Params& P, int sms, cudaStream_t st) {
   if (!P.xfold) return MDH_OK;
   const int64_t work = (int64_t)(P.nunits / P.ssplit) * t4::BM * t4::BN / 4;
   const unsigned g = (unsigned)std::max<int64_t>(1, std::min<int64_t>((work + 255) / 256, (int64_t)sms * 8));
-  t4::t4_xfold_kernel<<<g, 256, 0, st>>>(P);
+  // programmatic dependent launch: the fold's launch overlaps the GEMM's tail
+  cudaLaunchConfig_t cfg = {};
+  cfg.gridDim = dim3(g);
+  cfg.blockDim = dim3(256);
+  cfg.stream = st;
+  cudaLaunchAttribute attr[1];
+  attr[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+  attr[0].val.programmaticStreamSerializationAllowed = 1;
+  cfg.attrs = attr;
+  cfg.numAttrs = 1;
+  MDH_CUDA(cudaLaunchKernelEx(&cfg, t4::t4_xfold_kernel, P));
   return post_launch("t4_xfold_kernel");
 }
 
