@@ -1870,7 +1870,8 @@ mdh_status prepare_t4(Plan* p) {
       // few tiles, deep K (MCC conv5_1 at the paper's N = 1: 2 tiles × 72 k-blocks): split
       // every tile along K over the idle SMs, all splits write partials, and a separate
       // grid-wide fold (t4_xfold_kernel) adds them in split order
-      S = std::min({sms / T, P.num_kb / 4, t4::MAX_TAIL_UNITS1 / T});
+      // (auto: at least 4 k-blocks per split; a forced split=S may go down to one)
+      S = std::min({sms / T, p->tiles.split > 1 ? P.num_kb : P.num_kb / 4, t4::MAX_TAIL_UNITS1 / T});
       if (p->tiles.split > 1) S = std::min(S, p->tiles.split);
       if (S >= 2) {
         P.xfold = 1;
