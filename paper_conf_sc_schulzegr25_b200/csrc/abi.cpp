@@ -336,12 +336,13 @@ mdh_status mdh_stencil_sweeps(mdh_plan_t plan, void* u, void* v, int32_t sweeps,
     const int s = t & 1, d = s ^ 1;
     const void* in[1] = {buf[s]};
     void* out[1] = {buf[d]};
-    if (world > 1 && !nccl) {
-      // peer transport: the 7-point kernel stores its first / last plane straight into the
-      // neighbours' halo planes as well (one kernel per sweep, no copies)
+    if (world == 1 || !nccl) {
+      // one 7-point kernel per sweep, sweep t > 0 launched as a programmatic dependent of
+      // sweep t-1; peer transport: the kernel also stores its first / last plane straight
+      // into the neighbours' halo planes (no copies)
       mdh::reset_launch_count();
-      mdh_status e = mdh::launch_t1_halo(p, buf[s], buf[d], rank > 0 ? halo->peer_lo[d] : nullptr,
-                                         rank < world - 1 ? halo->peer_hi[d] : nullptr, st);
+      mdh_status e = mdh::launch_t1_halo(p, buf[s], buf[d], world > 1 && rank > 0 ? halo->peer_lo[d] : nullptr,
+                                         world > 1 && rank < world - 1 ? halo->peer_hi[d] : nullptr, st, t > 0);
       if (e == MDH_OK) {
         launches += mdh::launch_count();
         continue;

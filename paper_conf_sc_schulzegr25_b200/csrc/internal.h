@@ -155,7 +155,8 @@ mdh_status prepare_t0(Plan* p);
 mdh_status launch_t0(const Plan& p, const void* const* in, void* const* out, void* ws, cudaStream_t st);
 mdh_status prepare_t1(Plan* p);
 mdh_status launch_t1(const Plan& p, const void* const* in, void* const* out, void* ws, cudaStream_t st);
-mdh_status launch_t1_halo(const Plan& p, const void* in, void* out, void* hlo, void* hhi, cudaStream_t st);
+mdh_status launch_t1_halo(const Plan& p, const void* in, void* out, void* hlo, void* hhi, cudaStream_t st,
+                          bool pdl = false);
 mdh_status prepare_t2(Plan* p);
 mdh_status launch_t2(const Plan& p, const void* const* in, void* const* out, void* ws, cudaStream_t st);
 mdh_status prepare_t3(Plan* p);

@@ -139,6 +139,11 @@ __device__ __forceinline__ void rowq(const float* p, bool full, int64_t rem, flo
 // NX: x outputs per thread (4, or 8 with tile knob vec=8)
 template <bool VEC_IN, int VEC_OUT, int NX, int PF = 0>
 __global__ void __launch_bounds__(128) t1_j3d7_kernel(const __grid_constant__ J7Params P) {
+  // stencil time-stepping launches sweep t+1 as a programmatic dependent of sweep t: wait
+  // for the previous sweep's writes (a no-op for a plain launch), then let the next sweep's
+  // blocks be scheduled as this grid's SM slots free up
+  asm volatile("griddepcontrol.wait;" ::: "memory");
+  asm volatile("griddepcontrol.launch_dependents;" ::: "memory");
   const int x0 = (blockIdx.x * blockDim.x + threadIdx.x) * NX;
   const int y = blockIdx.y * blockDim.y + threadIdx.y;
   if (x0 >= P.X || y >= P.Y) return;
@@ -436,7 +441,7 @@ mdh_status prepare_t1(Plan* p) {
 }
 
 static mdh_status launch_j3d7(const Plan& p, const void* const* in, void* const* out, cudaStream_t st,
-                              void* hlo = nullptr, void* hhi = nullptr) {
+                              void* hlo = nullptr, void* hhi = nullptr, bool pdl = false) {
   J7Params P;
   memset(&P, 0, sizeof(P));
   P.hlo = (float*)hlo;
@@ -480,12 +485,13 @@ static mdh_status launch_j3d7(const Plan& p, const void* const* in, void* const*
   // 256 B 204.8 (5212 GB/s; 8 sweeps 1.740 -> 1.732 ms); the z+1 row loaded one step ahead
   // (software pipeline along z, +8 registers) 206.9, with the 256 B hint 206.8 — dropped
   const int pf = p.tiles.l2pf;
-#define J7(VI, VO)                                                                 \
-  do {                                                                             \
-    if (nx == 8) t1_j3d7_kernel<VI, VO, 8><<<grid, block, 0, st>>>(P);            \
-    else if (pf == 2) t1_j3d7_kernel<VI, VO, 4, 2><<<grid, block, 0, st>>>(P);    \
-    else if (pf == 1) t1_j3d7_kernel<VI, VO, 4, 1><<<grid, block, 0, st>>>(P);    \
-    else t1_j3d7_kernel<VI, VO, 4><<<grid, block, 0, st>>>(P);                    \
+  void (*kern)(J7Params) = nullptr;
+#define J7(VI, VO)                                              \
+  do {                                                          \
+    if (nx == 8) kern = t1_j3d7_kernel<VI, VO, 8>;              \
+    else if (pf == 2) kern = t1_j3d7_kernel<VI, VO, 4, 2>;      \
+    else if (pf == 1) kern = t1_j3d7_kernel<VI, VO, 4, 1>;      \
+    else kern = t1_j3d7_kernel<VI, VO, 4>;                      \
   } while (0)
   if (vin && vout) J7(true, 1);
   else if (vin && vodd) J7(true, 2);
@@ -493,20 +499,34 @@ static mdh_status launch_j3d7(const Plan& p, const void* const* in, void* const*
   else if (vout) J7(false, 1);
   else J7(false, 0);
 #undef J7
+  if (pdl) {                // time-stepping: a programmatic dependent of the previous sweep
+    cudaLaunchConfig_t cfg = {};
+    cfg.gridDim = grid;
+    cfg.blockDim = block;
+    cfg.stream = st;
+    cudaLaunchAttribute attr[1];
+    attr[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+    attr[0].val.programmaticStreamSerializationAllowed = 1;
+    cfg.attrs = attr;
+    cfg.numAttrs = 1;
+    MDH_CUDA(cudaLaunchKernelEx(&cfg, kern, P));
+  } else {
+    kern<<<grid, block, 0, st>>>(P);
+  }
   return post_launch("t1_j3d7_kernel");
 }
 
 // one sweep of a same-shape stencil plan with the halo stores fused into the 7-point
 // kernel (mdh_stencil_sweeps, peer transport); UNSUPPORTED when the plan does not run the
 // 7-point kernel or its first output plane is not buffer plane 1 (the caller then copies)
-mdh_status launch_t1_halo(const Plan& p, const void* in, void* out, void* hlo, void* hhi, cudaStream_t st) {
+mdh_status launch_t1_halo(const Plan& p, const void* in, void* out, void* hlo, void* hhi, cudaStream_t st, bool pdl) {
   if (p.tmpl != T1_STENCIL || p.auxi.empty() || p.auxi[0] == -2) return MDH_ERR_UNSUPPORTED;
   const Access& O = p.out[0].acc[0];
   const int dz = (int)p.auxi[0];
   if (O.L[dz] <= 0 || O.base < O.L[dz] || O.base >= 2 * O.L[dz]) return MDH_ERR_UNSUPPORTED;
   const void* ins[1] = {in};
   void* outs[1] = {out};
-  return launch_j3d7(p, ins, outs, st, hlo, hhi);
+  return launch_j3d7(p, ins, outs, st, hlo, hhi, pdl);
 }
 
 mdh_status launch_t1(const Plan& p, const void* const* in, void* const* out, void*, cudaStream_t st) {
