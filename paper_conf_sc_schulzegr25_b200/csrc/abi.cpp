@@ -145,7 +145,16 @@ static mdh_status execute_sharded(const mdh::Plan& p, const void* const* in, voi
   const bool float_allreduce = (p.flags & MDH_PLAN_FLOAT_ALLREDUCE) && p.n_out == 1 && p.f != MDH_F_PRL_COMPARE &&
                                p.redop == MDH_PW_ADD && (p.out[0].dtype == MDH_F32 || p.out[0].dtype == MDH_F64);
   if (exact_any_order || float_allreduce) {
-    return comm_allreduce(p.comm, lout[0], out[0], (size_t)p.out[0].elems, p.out[0].dtype, p.redop, st);
+    // the reduction runs over the whole output buffer; elements outside the output image
+    // must stay untouched (reading C-5), so reduce straight into out[0] only when the
+    // (injective) image covers it, else in place in the workspace and place the image
+    // with the S = 1 combine
+    const bool covers = p.out[0].nacc == 1 && p.Ncc == p.out[0].elems;
+    if (covers)
+      return comm_allreduce(p.comm, lout[0], out[0], (size_t)p.out[0].elems, p.out[0].dtype, p.redop, st);
+    MDH_TRY(comm_allreduce(p.comm, lout[0], lout[0], (size_t)p.out[0].elems, p.out[0].dtype, p.redop, st));
+    const void* one[1] = {lout[0]};
+    return launch_combine(p, one, 1, out, st);
   }
   MDH_TRY(comm_allgather(p.comm, local, gathered, per, st));
   const void* parts[MDH_MAX_WORLD * MDH_MAX_BUFS];
@@ -316,6 +325,11 @@ mdh_status mdh_stencil_sweeps(mdh_plan_t plan, void* u, void* v, int32_t sweeps,
     set_error("stencil sweeps: input and output buffers must have the same dtype and shape (rank >= 2)");
     return MDH_ERR_INVALID_ARG;
   }
+  {  // alignment and aliasing of u / v (reading C-27), as mdh_execute checks them
+    const void* ins[1] = {u};
+    void* outs[1] = {v};
+    MDH_TRY(mdh::check_ptrs(p, ins, outs));
+  }
   const int64_t nz = I.shape[0];
   const size_t plane = (size_t)(I.elems / nz) * mdh::dtype_size(I.dtype);
   const int world = halo ? halo->world : 1, rank = halo ? halo->rank : 0;
@@ -327,6 +341,34 @@ mdh_status mdh_stencil_sweeps(mdh_plan_t plan, void* u, void* v, int32_t sweeps,
         (rank < world - 1 && (!halo->peer_hi[0] || !halo->peer_hi[1]))) {
       set_error("stencil sweeps: world > 1 needs nccl_comm or the neighbours' halo-plane addresses");
       return MDH_ERR_INVALID_ARG;
+    }
+    // the peer transport has no cross-rank wait: sweep t+1 would read halo planes the
+    // neighbours' sweep t has not written yet, so the caller steps the ranks one sweep
+    // per call in lock-step
+    if (sweeps > 1) {
+      set_error("stencil sweeps: the peer transport runs one sweep per call (lock-step); use nccl_comm for more");
+      return MDH_ERR_INVALID_ARG;
+    }
+    const size_t esz = mdh::dtype_size(I.dtype);
+    for (int k = 0; k < 2; ++k) {
+      const void* q[2] = {halo->peer_lo[k], halo->peer_hi[k]};
+      for (const void* a : q)
+        if (a && reinterpret_cast<uintptr_t>(a) % esz) {
+          set_error("stencil sweeps: a peer halo-plane address is not %zu-byte aligned", esz);
+          return MDH_ERR_INVALID_ARG;
+        }
+      // a neighbour's halo plane must not lie inside this rank's own u / v
+      for (const void* a : q) {
+        if (!a) continue;
+        const uintptr_t h0 = (uintptr_t)a, h1 = h0 + plane;
+        for (const void* b : {(const void*)u, (const void*)v}) {
+          const uintptr_t b0 = (uintptr_t)b, b1 = b0 + (uintptr_t)I.elems * esz;
+          if (h0 < b1 && b0 < h1) {
+            set_error("stencil sweeps: a peer halo plane overlaps this rank's u or v");
+            return MDH_ERR_INVALID_ARG;
+          }
+        }
+      }
     }
   }
   cudaStream_t st = (cudaStream_t)cuda_stream;

@@ -132,15 +132,20 @@ mdh_status comm_halo_exchange(void* comm, int rank, int world, char* buf, size_t
   }
   ncclComm_t c = (ncclComm_t)comm;
   MDH_TRY(chk(g_nccl.groupStart(), "ncclGroupStart"));
+  // record the first failure but always close the group: an open group would capture
+  // this thread's later NCCL calls
+  mdh_status e = MDH_OK;
+  auto step = [&e](mdh_status s) { if (e == MDH_OK) e = s; };
   if (rank > 0) {
-    MDH_TRY(chk(g_nccl.send(buf + plane_bytes, plane_bytes, ncclUint8, rank - 1, c, st), "ncclSend"));
-    MDH_TRY(chk(g_nccl.recv(buf, plane_bytes, ncclUint8, rank - 1, c, st), "ncclRecv"));
+    step(chk(g_nccl.send(buf + plane_bytes, plane_bytes, ncclUint8, rank - 1, c, st), "ncclSend"));
+    step(chk(g_nccl.recv(buf, plane_bytes, ncclUint8, rank - 1, c, st), "ncclRecv"));
   }
   if (rank < world - 1) {
-    MDH_TRY(chk(g_nccl.send(buf + (nz - 2) * plane_bytes, plane_bytes, ncclUint8, rank + 1, c, st), "ncclSend"));
-    MDH_TRY(chk(g_nccl.recv(buf + (nz - 1) * plane_bytes, plane_bytes, ncclUint8, rank + 1, c, st), "ncclRecv"));
+    step(chk(g_nccl.send(buf + (nz - 2) * plane_bytes, plane_bytes, ncclUint8, rank + 1, c, st), "ncclSend"));
+    step(chk(g_nccl.recv(buf + (nz - 1) * plane_bytes, plane_bytes, ncclUint8, rank + 1, c, st), "ncclRecv"));
   }
-  return chk(g_nccl.groupEnd(), "ncclGroupEnd");
+  const mdh_status g = chk(g_nccl.groupEnd(), "ncclGroupEnd");
+  return e != MDH_OK ? e : g;
 }
 
 }  // namespace mdh

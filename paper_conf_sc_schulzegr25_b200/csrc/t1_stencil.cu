@@ -187,14 +187,16 @@ __global__ void __launch_bounds__(128) t1_j3d7_kernel(const __grid_constant__ J7
       for (int j = 0; j < NX; ++j)
         if (x0 + j < P.X) po[j] = o[j];
     }
-    float* ph = z == 0 ? P.hlo : (z == P.Z - 1 ? P.hhi : nullptr);
-    if (ph) {                      // this plane is also a neighbour's halo plane
-      ph += P.hbase + x0 + (int64_t)y * P.oLy;
+    // this plane may also be a neighbour's halo plane: the first owned plane goes to the
+    // lower neighbour, the last to the upper one (a one-plane slab feeds both); the two
+    // stores are independent, so a rank with only one neighbour still writes its halo
+    if (z == 0 && P.hlo) {
+      float* q = P.hlo + P.hbase + x0 + (int64_t)y * P.oLy;
 #pragma unroll
       for (int j = 0; j < NX; ++j)
-        if (x0 + j < P.X) ph[j] = o[j];
+        if (x0 + j < P.X) q[j] = o[j];
     }
-    if (P.hlo && P.hhi && P.Z == 1) {   // a one-plane slab feeds both neighbours
+    if (z == P.Z - 1 && P.hhi) {
       float* q = P.hhi + P.hbase + x0 + (int64_t)y * P.oLy;
 #pragma unroll
       for (int j = 0; j < NX; ++j)

@@ -154,3 +154,31 @@ def test_tile_override_and_table(mdh, tmp_path):
     assert d["tiles"]["split"] == 33 and d["tiles"]["source"].startswith("table")
     d = mdh.Plan(S.dot(1 << 22, "f32"), tile_table=str(t)).describe()   # nearest bucket
     assert d["tiles"]["split"] == 33
+
+
+def test_sweeps_argument_checks_on_host(mdh):
+    """mdh_stencil_sweeps validates its pointers before enqueueing anything (no GPU needed):
+    u == v or overlapping u/v (reading C-27), a pointer that is not 16-byte aligned, and
+    the peer transport asked for more than one sweep per call (it has no cross-rank wait)
+    are INVALID_ARG."""
+    q = mdh.Plan(S.jacobi3d_sweep(10, 10, 10))
+    L = mdh.lib()
+    n = 10 * 10 * 10 * 4
+    base = 1 << 32
+
+    def call(u, v, sweeps=1, halo=None):
+        res = ctypes.c_int32()
+        return L.mdh_stencil_sweeps(q._h, u, v, sweeps, ctypes.byref(halo) if halo else None,
+                                    None, 0, None, ctypes.byref(res))
+
+    INVALID_ARG = 1
+    assert call(base, base) == INVALID_ARG                       # u is v
+    assert call(base, base + n // 2) == INVALID_ARG              # overlap
+    assert call(base + 4, base + 2 * n) == INVALID_ARG           # misaligned u
+    assert call(base, base + 2 * n + 8) == INVALID_ARG           # misaligned v
+    h = mdh.Halo()
+    h.rank, h.world = 0, 2
+    h.peer_hi[0], h.peer_hi[1] = base + 8 * n, base + 9 * n
+    assert call(base, base + 2 * n, sweeps=2, halo=h) == INVALID_ARG   # peer: one sweep per call
+    h.peer_hi[1] = base + n                                      # a "peer" plane inside own v
+    assert call(base, base + n, sweeps=1, halo=h) == INVALID_ARG

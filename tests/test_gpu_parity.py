@@ -273,7 +273,41 @@ def test_prl_ties_full(R):
         assert_close_full(spec, ins, got, 0, kind="exact")
 
 
-@pytest.mark.parametrize("NI", [(1 << 20, 1 << 14), (1 << 14, 1 << 20)])
+# field codes around the fp16 edges of the packed compare (t5_prl.cu: code x is held as the
+# fp16 pattern x < 0x7C00 ? x : x + 0x401): +0, subnormals, the first normal, the largest
+# finite code, the codes remapped past the NaN range, and the last packable code
+PRL_EDGE_CODES = np.array([0, 1, 2, 0x3FF, 0x400, 0x401, 0x7BFF, 0x7C00, 0x7C01, 0x7E00, 0x7FFF], np.uint32)
+
+
+@pytest.mark.parametrize("case", ["edges_packed", "db_tile_unpackable", "new_unpackable", "all_unpackable"])
+@pytest.mark.parametrize("op", ["PW_PRL_ARGMAX", "PW_PRL_PAPER"])
+def test_prl_packed_and_general_paths(case, op):
+    """Bit-exact on codes chosen to trip the packed fp16 compare (many agreements among
+    the edge codes), and on inputs that force the per-field u32 compares: one DB tile with
+    a code >= 2^15 (that tile alone, mid-fold), one new record with 0xFFFFFFFF (its whole
+    CTA), and every code >= 2^15 (codes differing only above bit 15 must not agree)."""
+    N, I = 1500, 1700
+    ins = G.prl_inputs(N, I, seed_base=5700)
+    g = np.random.Generator(np.random.PCG64(5799))
+    for k in range(8):
+        for b in (k, 8 + k):
+            n = len(ins[b])
+            pick = g.random(n) < 0.5
+            ins[b] = np.where(pick, PRL_EDGE_CODES[g.integers(0, len(PRL_EDGE_CODES), n)], ins[b]).astype(np.uint32)
+    if case == "db_tile_unpackable":
+        ins[8 + 3][600] = 0x8000                      # DB tile 1 (records 512..1023)
+    elif case == "new_unpackable":
+        ins[5][1] = 0xFFFFFFFF
+    elif case == "all_unpackable":
+        for b in range(16):
+            ins[b] = (ins[b] | np.uint32(0x10000) * (g.integers(0, 2, len(ins[b])).astype(np.uint32) + 1)).astype(np.uint32)
+    spec = S.prl(N, I, op)
+    got, p = run_gpu(spec, ins)
+    assert p.template == "T5_prl_pairwise"
+    assert_close_full(spec, ins, got, 0, kind="exact")
+
+
+@pytest.mark.parametrize("NI", [(1 << 20, 1 << 14), (1 << 14, 1 << 20), (1 << 15, 1 << 15)])
 def test_prl_config_sampled(NI):
     N, I = NI
     ins = G.prl_inputs(N, I, seed_base=5000)

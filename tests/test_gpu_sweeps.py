@@ -41,17 +41,18 @@ def test_sweeps_whole_domain(zyx, T):
     assert err.max() <= 1e-4, err.max()
 
 
-@pytest.mark.parametrize("world", [2, 3, 5])
-def test_sweeps_zsharded_virtual_ranks(world):
+@pytest.mark.parametrize("Z,world", [(23, 2), (23, 3), (23, 5), (7, 5), (5, 3)])
+def test_sweeps_zsharded_virtual_ranks(Z, world):
     """Slabs with one halo plane per side, a sweep per call in lock-step on one stream; after
     each sweep a rank's first / last owned plane is copied into the neighbours' halo planes
     (mdh_halo peer transport).  The owned planes equal the whole-domain GPU run bit for bit
     (same per-point arithmetic) and the fp64 oracle within the scale-normalised 1e-4.  The
     7-point kernel stores its first / last plane into the neighbours' halos itself (one
-    launch per sweep)."""
+    launch per sweep).  Z = 7 / 5 give one-plane slabs (nz = 3) at every rank, rank 0 and
+    the last rank included, whose single plane feeds one or both neighbours."""
     import torch
     from paper_conf_sc_schulzegr25_b200 import Halo, Plan
-    Z, Y, X, T = 23, 12, 40, 4
+    Y, X, T = 12, 40, 4
     u0 = _field(Z, Y, X, 3420)
     whole = Plan(S.jacobi3d_sweep(Z, Y, X))
     wu = torch.from_numpy(u0).cuda()
@@ -102,6 +103,8 @@ def test_sweeps_rejects_bad_plans():
     h.rank, h.world = 1, 2                           # no transport given
     with pytest.raises(MdhError):
         q.stencil_sweeps(u, u.clone(), 1, halo=h)
+    with pytest.raises(MdhError):                    # u is v: aliasing (reading C-27)
+        q.stencil_sweeps(u, u, 1)
 
 
 def _box3_sweep(Y, X):
