@@ -96,6 +96,14 @@ def workload(name, world=1, rank=0):
         spec = S.mcc(256, 7, 7, 512, 3, 3, 512, "bf16")
         return dict(spec=spec, inputs=lambda: G.mcc_inputs(spec), work=2.0 * 256 * 49 * 512 * 4608, unit="TFLOP/s",
                     scale=1e12, bound="tensor", dtype="bf16", desc="MCC ResNet-50 conv5_1 3x3/s2 N=256 bf16")
+    if name == "mcc_conv1_bf16":
+        # C4b-B (reading C-21): conv1 7x7/s2, C=3, K=64, P=Q=112 at N=256 — HBM-bound on its
+        # 822 MB fp32 output (bytes: image + filter read once, output written once)
+        spec = S.mcc(256, 112, 112, 64, 7, 7, 3, "bf16")
+        byts = 2.0 * 256 * 230 * 230 * 3 + 2.0 * 64 * 147 + 4.0 * 256 * 112 * 112 * 64
+        return dict(spec=spec, inputs=lambda: G.mcc_inputs(spec), work=byts, unit="GB/s", scale=1e9, bound="hbm",
+                    dtype="bf16", flops=2.0 * 256 * 112 * 112 * 64 * 147,
+                    desc="MCC ResNet-50 conv1 7x7/s2 N=256 bf16->fp32 (Fig 3 MCC Inp.2; HBM-bound on the 822 MB output)")
     if name == "mcc_bf16_n1":
         spec = S.mcc(1, 7, 7, 512, 3, 3, 512, "bf16")
         return dict(spec=spec, inputs=lambda: G.mcc_inputs(spec), work=2.0 * 49 * 512 * 4608, unit="TFLOP/s",
@@ -134,7 +142,7 @@ def workload(name, world=1, rank=0):
 
 
 SUITE = ["dot_f32", "dot_i32", "dot_f32_2^28", "matvec_f32", "matvec_4096", "jacobi3d", "jacobi3d_sweeps8", "gaussian2d", "matmul_f32",
-         "matmul_bf16", "ccsd_bf16", "mcc_bf16", "mcc_bf16_n1", "mcc_caps_bf16", "prl_A", "prl_B", "prefix_sum_f32", "mbbs_f32"]
+         "matmul_bf16", "ccsd_bf16", "mcc_bf16", "mcc_conv1_bf16", "mcc_bf16_n1", "mcc_caps_bf16", "prl_A", "prl_B", "prefix_sum_f32", "mbbs_f32"]
 
 
 def roofline(w, seconds, pk):

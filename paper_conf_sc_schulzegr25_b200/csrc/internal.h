@@ -164,6 +164,9 @@ mdh_status launch_t3(const Plan& p, const void* const* in, void* const* out, voi
 mdh_status prepare_t4(Plan* p);
 mdh_status launch_t4(const Plan& p, const void* const* in, void* const* out, void* ws, cudaStream_t st);
 bool t4_supported(const Plan& p, std::string* why);
+// T4 small-K direct contraction (t4_conv.cu): true if the plan was set up for it
+bool prepare_t4_conv(Plan* p);
+mdh_status launch_t4_conv(const Plan& p, const void* const* in, void* const* out, cudaStream_t st);
 mdh_status prepare_t5(Plan* p);
 mdh_status launch_t5(const Plan& p, const void* const* in, void* const* out, void* ws, cudaStream_t st);
 mdh_status prepare_t6(Plan* p);

@@ -1687,6 +1687,7 @@ static bool plan_im2col(const Plan* p, T4State* s) {
 mdh_status prepare_t4(Plan* p) {
   std::string why;
   if (!t4_supported(*p, &why)) { set_error("T4: %s", why.c_str()); return MDH_ERR_UNSUPPORTED; }
+  if (prepare_t4_conv(p)) return MDH_OK;           // small-K direct variant (t4_conv.cu)
   const Contraction& c = p->con;
   T4State* s = new T4State();
   size_t ws = 0;
@@ -2096,6 +2097,7 @@ static mdh_status run_permute(const t4::Layout2D& L, const uint16_t* src, char* 
 }
 
 mdh_status launch_t4(const Plan& p, const void* const* in, void* const* out, void* ws, cudaStream_t st) {
+  if (p.t4_variant == 1024) return launch_t4_conv(p, in, out, st);
   const char* dc = nullptr;
   MDH_TRY(device_consts(p, &dc));
   const T4State* s = (const T4State*)p.tmaps;

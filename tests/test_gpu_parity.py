@@ -569,6 +569,33 @@ def test_t4_few_tile_splitk(shape, out):
     assert np.array_equal(got[0], got2[0])
 
 
+@pytest.mark.parametrize("cfg", [(1, 9, 13, 64, 7, 7, 3), (3, 17, 19, 64, 7, 7, 3), (2, 112, 112, 64, 7, 7, 3),
+                                 (2, 20, 21, 64, 3, 3, 3)])
+def test_mcc_small_k_direct(cfg):
+    """MCC with C = 3 (conv1 7×7/s2, Fig 3 MCC Inp.2 P:529, reading C-21; and a 3×3 layer) on
+    the small-K direct kernel (t4_conv.cu): A rows built in TMEM from staged input runs.
+    Ragged last tiles (M = 117, 969) and tiles straddling two images (P·Q = 323) included;
+    full comparison with the fp64 oracle on the same bf16 inputs."""
+    spec = S.mcc(*cfg, dtype="bf16")
+    x = G.mcc_inputs(spec)
+    got, p = run_gpu(spec, x)
+    assert p.template == "T4_tcgen05_contraction"
+    assert p.describe()["t4_variant"] == 1024, p.describe()
+    assert_close_full(spec, x, got, 1e-2, kind="scale")
+
+
+def test_mcc_conv1_config_sampled():
+    """conv1 7×7/s2 at N = 256 (C4b-B): 20 000 sampled outputs, each
+    folded over its full 147-term window by the oracle; plus determinism (bit-identical rerun)."""
+    spec = S.mcc(256, 112, 112, 64, 7, 7, 3, "bf16")
+    x = G.mcc_inputs(spec)
+    got, p = run_gpu(spec, x)
+    assert p.describe()["t4_variant"] == 1024
+    assert_close_points(spec, x, got, 1e-2, n=20000, kind="scale")
+    got2, _ = run_gpu(spec, x, plan=p)
+    assert np.array_equal(got[0], got2[0])
+
+
 def test_mcc_bf16_config_sampled():
     spec = S.mcc(256, 7, 7, 512, 3, 3, 512, "bf16")
     x = G.mcc_inputs(spec)

@@ -38,6 +38,9 @@ def cases():
         "t4_cl4": (lambda: S.matmul(700, 1000, 512, "bf16"), "positive", "cluster=4"),
         "t1_sweep": (lambda: S.jacobi3d_sweep(12, 10, 70), "positive", None),
         "t4_ag4": (lambda: S.mcc_caps(2, 5, 3, 4, 3, 3, 3, dtype="bf16"), "positive", None),
+        "t4_conv": (lambda: S.mcc(3, 17, 19, 64, 7, 7, 3, "bf16"), "positive", None),
+        "t4_conv_ns3": (lambda: S.mcc(3, 17, 19, 64, 7, 7, 3, "bf16"), "positive", "stages=3"),
+        "t4_conv3x3": (lambda: S.mcc(2, 20, 21, 64, 3, 3, 3, "bf16"), "positive", None),
         "t6_colfold": (lambda: S.mbbs(300, 1000), "positive", None),
         "t5": (lambda: S.prl(300, 2000), "prl", None),
         "t6": (lambda: S.prefix_sum([3, 9000], 1), "positive", None),
