@@ -51,7 +51,8 @@ typedef enum {
   MDH_ERR_INVALID_SPEC = 2,  /* malformed: out-of-bounds access, non-injective output,  */
                              /* size 0, f arity mismatch, declared shape too small      */
   MDH_ERR_UNSUPPORTED = 3,   /* valid MDH but outside this build's catalog: mixed pw    */
-                             /* operators (C-3), unknown f/dtype combination, ps (NEXT)  */
+                             /* operators (C-3), unknown f/dtype combination, sharding */
+                             /* a ps dim                                                */
   MDH_ERR_OUT_OF_MEMORY = 4,
   MDH_ERR_CUDA = 5,          /* a CUDA runtime/driver call or a kernel launch failed    */
   MDH_ERR_NCCL = 6,          /* NCCL missing or an NCCL call failed                     */
@@ -142,7 +143,10 @@ typedef struct {
   int32_t world_size;    /* 1 ⇒ single GPU                                             */
   int32_t rank;
   void* nccl_comm;       /* from mdh_comm_init, or NULL (VIRTUAL_SHARD / world 1)       */
-  int32_t shard_dim;     /* -1 ⇒ the planner chooses                                   */
+  int32_t shard_dim;     /* -1 ⇒ the planner chooses (world_size > 1).  world_size 1
+                            with nccl_comm and shard_dim >= 0: a one-rank shard that runs
+                            the sharded execute path (collective over the one-rank
+                            communicator) — the NCCL data plane on one GPU              */
   uint32_t flags;
   const char* tile_table;/* path of a tile table JSON; NULL ⇒ $MDH_TILE_TABLE, else the */
                          /* table compiled into the library                             */

@@ -239,7 +239,7 @@ mdh_status mdh_execute(mdh_plan_t plan, const void* const* in, void* const* out,
   }
   cudaStream_t st = (cudaStream_t)cuda_stream;
   try {
-    if (p.world > 1 && p.shard_is_red && p.comm && !(p.flags & MDH_PLAN_NO_COLLECTIVE))
+    if (p.sharded && p.shard_is_red && p.comm && !(p.flags & MDH_PLAN_NO_COLLECTIVE))
       return mdh::execute_sharded(p, in, out, (char*)workspace, st);
     return mdh::run_template(p, in, out, workspace, st);
   } catch (...) {

@@ -102,6 +102,7 @@ struct Plan {
   int device = 0, world = 1, rank = 0, shard_dim = -1;
   uint32_t flags = 0;
   void* comm = nullptr;
+  bool sharded = false;               // the shard rewrite ran (world > 1, or a one-rank NCCL shard)
   bool shard_is_red = false;
   int64_t shard_start = 0, shard_len = 0, global_size = 0;
   // ---- workspace ----

@@ -460,7 +460,10 @@ mdh_status build_plan(const mdh_spec* spec, const mdh_plan_opts* opts, Plan* p) 
     set_error("rank %d / world %d invalid", p->rank, p->world);
     return MDH_ERR_INVALID_ARG;
   }
-  if (p->world > 1) {
+  // a one-rank plan with a communicator and an explicit shard dim runs the sharded path too
+  // (its collective over the one-rank NCCL communicator): the NCCL data plane on one GPU
+  if (p->world > 1 || (p->comm && opts->shard_dim >= 0)) {
+    p->sharded = true;
     int sd = opts->shard_dim >= 0 ? opts->shard_dim : choose_shard_dim(*p);
     if (sd < 0 || sd >= p->D) { set_error("no dimension can be sharded over %d ranks", p->world); return MDH_ERR_INVALID_ARG; }
     if (p->size[sd] < p->world) { set_error("shard dim %d has %lld < %d points", sd, (long long)p->size[sd], p->world); return MDH_ERR_INVALID_ARG; }
@@ -493,7 +496,7 @@ mdh_status build_plan(const mdh_spec* spec, const mdh_plan_opts* opts, Plan* p) 
   }
   // pw shard: room for the gathered partials of all ranks
   p->ws_comm = 0;
-  if (p->world > 1 && p->shard_is_red && p->comm && !(p->flags & MDH_PLAN_NO_COLLECTIVE)) {
+  if (p->sharded && p->shard_is_red && p->comm && !(p->flags & MDH_PLAN_NO_COLLECTIVE)) {
     size_t per = 0;
     for (int b = 0; b < p->n_out; ++b) per += ((size_t)p->out[b].elems * dtype_size(p->out[b].dtype) + 255) / 256 * 256;
     p->ws_comm = per * (size_t)(p->world + 1);

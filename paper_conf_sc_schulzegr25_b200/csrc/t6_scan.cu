@@ -4,22 +4,27 @@
 // One ps dim d_ps is kept and folded over [0, k]; other kept (cc) dims enumerate rows c;
 // pw(add) dims are folded completely.  Because every operator here is +, the result is
 //   R[c, k] = Σ_{t ≤ k} z[c, t],   z[c, t] = Σ_{pw} f(x(c, t, pw))
-// which the GPU evaluates as
-//   K1  z[c, t]          — one thread per (c, t), sequential fold over the pw dims
-//   K2  per (c, chunk)   — block inclusive scan of a 4096-element chunk (16 per thread,
-//                          warp shuffles, warps in order) + the chunk total
-//   K3  per row          — exclusive scan of the chunk totals (in chunk order)
-//   K4  per (c, t)       — R = local scan + chunk offset, written through out_view
-// (K3/K4 are skipped when a row fits one chunk).  Deterministic: fixed association order,
-// no atomics.  HBM-bound: z and the local scans are each written and read once.
+// Deterministic throughout (every sum in a fixed association order, no float atomics).
+// Three paths, chosen at plan time (prepare_t6):
 //
-// Long rows read straight from the input (no pw dims, f = IDENTITY, unit strides) take a
-// single persistent kernel instead (t6_seg_scan_kernel): the row is cut into L2-sized
-// segments; per segment every CTA (A) reduces its contiguous sub-range, (grid barrier)
-// (B) takes its exclusive prefix = carry + Σ of the lower CTAs' totals in CTA order, and
-// (C) re-scans its sub-range — now an L2 hit — writing the output, so HBM sees one read
-// and one write per element.  Still deterministic (every sum in a fixed order), unlike a
-// decoupled look-back whose association depends on timing.
+//  * Long unit-stride rows read straight from the input (no pw dims, f = IDENTITY) — the
+//    prefix sum of 2^26 fp32 — take ONE persistent streaming kernel (t6_stream_scan_kernel,
+//    the default): one CTA per SM owns a slice of every segment, brought into a shared-
+//    memory ring by TMA bulk copies issued three jobs ahead; each CTA publishes its slice
+//    total as a self-validating (tag, value) word, and its exclusive prefix is the carry
+//    plus the totals of the lower CTAs in CTA order (polled by warp 0, no grid barrier);
+//    the slice is scanned in place (per-thread sequential runs, warp/CTA scans in order)
+//    and written back with a bulk store — HBM sees one read and one write per element.
+//    (t6_seg_scan_kernel, a segmented variant with a grid barrier between a reduce and a
+//    re-scan pass, stays behind tile knob seg > 0 for measurements.)
+//  * One pw dim folded into a unit-stride ps dim in fp32 (MBBS) — the column fold
+//    (t6_colfold_kernel: 4 columns per thread with 16-byte loads, the rows split over
+//    blocks × 8 threads, folded in order by a per-column-group ticket), then the register
+//    row scan t6_rowscan4_kernel launched as a programmatic dependent (rows ≤ 8 × 4096).
+//  * Otherwise: K1 z[c, t] = the pw fold per (c, t) (t6_fold_kernel), K2 a block scan of
+//    each 4096-element chunk with its total (t6_chunk_scan_kernel, or one 1024-thread row
+//    scan for short rows), K3 an exclusive scan of the chunk totals (t6_sums_kernel), K4
+//    the chunk offsets added and the result written through out_view (t6_fix_kernel).
 #include <algorithm>
 #include <mutex>
 
