@@ -420,14 +420,14 @@ mdh_status prepare_t5(Plan* p) {
   p->tab_off[1] = add_const(p, W, sizeof(W));
   int64_t N = nd >= 0 ? p->size[nd] : 1, I = id >= 0 ? p->size[id] : 1;
   // 4 new records per thread (8: tile knob vec=8 — measured 1147 vs 1466 Gpairs/s on 2^20×2^14)
-  int Rn = T5_R;
-  const bool forced = p->tiles.source.find("forced") != std::string::npos;
-  if (forced && p->tiles.vec == 8) Rn = T5_R8;
+  // tile knobs (defaults in tiles.cpp): vec = new records per thread (4 | 8), stages = CTAs
+  // per SM the registers are budgeted for (2 | 3, R = 4 only), bk = DB-loop unroll (2 | 4 | 8).
+  // Measured (prl_A / prl_B, ms): R=4, 3 CTAs/SM, unroll ×4 7.40 / 7.47; 2 CTAs/SM
+  // 7.80 / 7.65; unroll ×2 8.04 (3 CTAs) / 8.64 (2 CTAs); ×8 7.90 / 8.37
+  const int Rn = p->tiles.vec == 8 ? T5_R8 : T5_R;
   p->tiles.vec = Rn;
-  // measured (prl_A / prl_B, ms): R=4 with 3 CTAs/SM and the DB loop unrolled ×4 7.40 / 7.47;
-  // 2 CTAs/SM 7.80 / 7.65; unroll ×2 8.04 (3 CTAs) / 8.64 (2 CTAs); ×8 7.90 / 8.37
-  p->tiles.stages = forced && p->tiles.stages == 2 ? 2 : (Rn == T5_R ? 3 : 2);
-  p->tiles.bk = forced && (p->tiles.bk == 2 || p->tiles.bk == 8) ? p->tiles.bk : 4;   // DB-loop unroll
+  p->tiles.stages = p->tiles.stages == 3 && Rn == T5_R ? 3 : 2;
+  p->tiles.bk = (p->tiles.bk == 2 || p->tiles.bk == 8) ? p->tiles.bk : 4;
   int64_t nblk = (N + T5_THREADS * Rn - 1) / (T5_THREADS * Rn);
   // split the DB dim when N alone gives less than two waves of CTAs, choosing S so the
   // CTAs fill whole waves: time ∝ ceil(nblk·S / slots) / S (slots = SMs × resident CTAs),

@@ -5,7 +5,7 @@
 #
 # steps (each bounded by its own timeout so a hang cannot eat the call):
 #   test[:<pytest -k expr>]           pytest -m gpu (all, or the -k selection)          -> tests.log
-#   time:<w1,w2,..>[@<force_tile>]    tools/time_one.py device timings (L2 flushed)     -> time.jsonl
+#   time:<w1+w2+..>[@<force_tile>]    tools/time_one.py device timings (L2 flushed)     -> time.jsonl
 #   ncu:<kernel regex>:<workload>     ncu --set full of one launch of the kernel        -> ncu_<workload>.ncu-rep
 #   launches[:<bench args>]           ncu launch list of a short bench run              -> launches.csv
 #   bench[:<bench args>]              python bench.py (default args)                    -> bench.json
@@ -34,7 +34,7 @@ for step in "$@"; do
     time)
       wl=${arg%%@*}; ft=""
       [ "$wl" != "$arg" ] && ft="--force-tile ${arg#*@}"
-      timeout 900 python tools/time_one.py ${wl//,/ } --reps 10 $ft >> "$OUT/time.jsonl" 2>> "$OUT/time.err"
+      timeout 900 python tools/time_one.py ${wl//+/ } --reps 10 $ft >> "$OUT/time.jsonl" 2>> "$OUT/time.err"
       tail -5 "$OUT/time.jsonl" ;;
     ncu)
       k=${arg%%:*}; wl=${arg#*:}

@@ -42,6 +42,17 @@ def cases():
         ("t4_mcc_bf16_conv5_1", lambda: (S.mcc(256, 7, 7, 512, 3, 3, 512, "bf16"),
                                          G.mcc_inputs(S.mcc(256, 7, 7, 512, 3, 3, 512, "bf16"))),
          ["bn=256", "bn=512", "bn=256,split=1", "bn=512,split=1"]),
+        # per-rank shapes of the strong-scaled configs (bench.py --gpus N):
+        # MatMul 4096³ on M at 2/4/8 GPUs, Jacobi3D 512³ z-slabs, PRL A/B DB slices
+        *[(f"rank_mm_bf16_{m}", (lambda m=m: (S.matmul(m, 4096, 4096, "bf16"), G.matmul_inputs(m, 4096, 4096, "bf16", "signed"))),
+           ["bn=256", "bn=512", "bn=256,split=2", "bn=512,split=2", "bn=256,split=1", "bn=512,split=1"])
+          for m in (2048, 1024, 512)],
+        *[(f"rank_jacobi3d_{z}", (lambda z=z: (S.jacobi3d(z, 512, 512), G.jacobi3d_inputs(z, 512, 512))),
+           [f"zchunk={c}" for c in (4, 8, 16, 32)]) for z in (257, 130, 66)],
+        *[(f"rank_prl_A_{i}", (lambda i=i: (S.prl(1 << 20, i), G.prl_inputs(1 << 20, i))),
+           [f"split={c}" for c in (1, 2, 3, 4)]) for i in (8192, 4096, 2048)],
+        *[(f"rank_prl_B_{i}", (lambda i=i: (S.prl(1 << 14, i), G.prl_inputs(1 << 14, i))),
+           [f"split={c}" for c in (9, 18, 27, 37, 48, 64)]) for i in (524288, 262144, 131072)],
         ("mcc_f32_n1", lambda: (S.mcc(1, 7, 7, 512, 3, 3, 512, "f32"),
                                 G.mcc_inputs(S.mcc(1, 7, 7, 512, 3, 3, 512, "f32"))),
          [f"split={s}" for s in (1, 8, 16, 32, 64, 72)]),
