@@ -457,6 +457,33 @@ def test_matmul_bf16_full_size():
     assert np.array_equal(got[0], G.bf16_bits_to_f32(x[1]))
 
 
+@pytest.mark.parametrize("M", [512, 1024, 2048])
+@pytest.mark.parametrize("dt", ["bf16", "f32"])
+def test_matmul_per_rank_shapes(M, dt):
+    """The per-rank shapes of MatMul 4096³ sharded on M over 8 / 4 / 2 GPUs,
+    each with the tiles the table holds for that bucket (bf16: stream-K narrow tiles at
+    M = 512), on T4 (bf16) and T3 (fp32): sampled points against the oracle, plus the
+    ones → K closed form."""
+    spec = S.matmul(M, 4096, 4096, dt)
+    x = G.matmul_inputs(M, 4096, 4096, dt, "signed")
+    got, p = run_gpu(spec, x)
+    assert p.template == ("T4_tcgen05_contraction" if dt == "bf16" else "T3_simt_contraction")
+    assert_close_points(spec, x, got, 1e-2 if dt == "bf16" else 1e-4, n=4000, kind="scale")
+    ones = G.matmul_inputs(M, 4096, 4096, dt, "ones")
+    got, _ = run_gpu(spec, ones, plan=p)
+    assert np.all(got[0] == 4096.0)
+
+
+def test_ccsd_paper_inp1_full():
+    """The paper's CCSD(T) Inp.1 reading (C-22) checked in FULL — every one of the 37.7 M
+    outputs against the fp64 oracle — in fp32 (T3) and bf16 (T4)."""
+    for dt, tol in (("f32", 1e-4), ("bf16", 1e-2)):
+        spec = S.ccsd_sd2(dtype=dt)
+        x = G.gen_inputs(spec, 4011)
+        got, _ = run_gpu(spec, x)
+        assert_close_full(spec, x, got, tol, kind="scale")
+
+
 def test_ccsd_bf16_tcgen05():
     # tiny brute-force size, the paper's Inp.1 reading (C-22), then the O=24/V=72 config sampled
     for spec, n in ((S.ccsd_sd1(2, 3, "bf16"), None), (S.ccsd_sd2(dtype="bf16"), 20000),

@@ -35,6 +35,21 @@ def test_mbbs_closed_form():
     assert np.array_equal(r, 10.0 * np.arange(1, 21))
 
 
+def test_mbbs_both_orientations():
+    """MBBS as (pw(add), ps(add)) over loops (i, j) and as (ps(add), pw(add)) over loops
+    (j, i) (SURVEY §8(f) F1's orientation): the same closed form R[j] = Σ_{j'≤j} Σ_i X[i,j']
+    — exactly for int32, and to fp64 rounding for floats (the fold orders differ)."""
+    X = G.rng(7).integers(-1000, 1000, (33, 29)).astype(np.int32)
+    ref = np.cumsum(X.astype(np.int64).sum(axis=0))
+    for order in ("pw_ps", "ps_pw"):
+        assert np.array_equal(oracle.evaluate(S.mbbs(33, 29, "i32", order), [X])[0], ref)
+    Xf = G.rng(8).uniform(-1, 1, (33, 29)).astype(np.float32)
+    a = oracle.evaluate(S.mbbs(33, 29, "f32", "pw_ps"), [Xf])[0]
+    b = oracle.evaluate(S.mbbs(33, 29, "f32", "ps_pw"), [Xf])[0]
+    exact = np.array([sum(float(v) for v in Xf[:, :j + 1].ravel()) for j in range(29)])
+    assert np.max(np.abs(a - exact)) < 1e-12 and np.max(np.abs(b - exact)) < 1e-12
+
+
 def test_ps_homomorphism_split():
     """Listing 17 for a contiguous split P|Q of the ps dim: res[P] = lhs, res[q] = lhs[max P] ⊕ rhs[q]."""
     n, s = 1000, 377
@@ -118,6 +133,23 @@ def test_gpu_mbbs(IJ):
         assert np.max(np.abs(got[0] - ref) / ref) <= 1e-4
     got2, _ = run_gpu(spec, x, plan=p)
     assert np.array_equal(got[0], got2[0])
+
+
+@gpu
+@pytest.mark.parametrize("IJ", [(64, 37), (1000, 5000), (8192, 8192)])
+def test_gpu_mbbs_ps_pw_orientation(IJ):
+    """MBBS with the loops swapped — md_hom[J,I](id, (ps(add), pw(add))) — against the
+    oracle (small) or the closed form (large)."""
+    from gpu_util import assert_close_full, run_gpu
+    spec = S.mbbs(*IJ, order="ps_pw")
+    x = G.gen_inputs(spec, 6250, "positive")
+    got, p = run_gpu(spec, x)
+    assert p.template == "T6_prefix_scan"
+    if IJ[0] * IJ[1] <= 64 * 64:
+        assert_close_full(spec, x, got, 1e-4, kind="rel")
+    else:
+        ref = np.cumsum(x[0].astype(np.float64).sum(axis=0))
+        assert np.max(np.abs(got[0] - ref) / ref) <= 1e-4
 
 
 @gpu
