@@ -277,6 +277,15 @@ int32_t mdh_last_launch_count(void);
  * returns n; 0 when tracing is off, -1 on a CUDA error.  `host` is caller-owned.         */
 int64_t mdh_debug_t4_trace(uint64_t* host, int64_t max_units);
 
+/* Diagnostics: measured instruction-throughput peaks of `device` (the roofline
+ * denominators of the pipe-bound templates): fp32 FFMA TFLOP/s (8 FFMA
+ * chains per thread), ALU-pipe thread-instructions/s (LOP3 chains) and the issue rate
+ * (thread-instructions/s: the best of the FFMA kernel and an FFMA/LOP3 interleave) — each
+ * the best of 3 ~ms launches
+ * of 4 × 256 threads per SM, timed with CUDA events.  Synchronises; any pointer may be
+ * NULL.  Errors: MDH_ERR_CUDA.                                                          */
+mdh_status mdh_measure_peaks(int32_t device, double* ffma_tflops, double* alu_tops, double* issue_tops);
+
 #ifdef __cplusplus
 }
 #endif

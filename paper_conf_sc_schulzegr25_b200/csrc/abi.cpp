@@ -430,6 +430,10 @@ mdh_status mdh_comm_init(const void* id128, int32_t world, int32_t rank, int32_t
 }
 mdh_status mdh_comm_destroy(void* comm) { return mdh::comm_destroy(comm); }
 
+mdh_status mdh_measure_peaks(int32_t device, double* ffma_tflops, double* alu_tops, double* issue_tops) {
+  return mdh::measure_peaks(device, ffma_tflops, alu_tops, issue_tops);
+}
+
 const char* mdh_last_error(void) { return mdh::g_err.c_str(); }
 int32_t mdh_abi_version(void) { return MDH_ABI_VERSION; }
 int32_t mdh_last_launch_count(void) { return mdh::launch_count(); }

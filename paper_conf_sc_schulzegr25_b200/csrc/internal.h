@@ -174,6 +174,9 @@ mdh_status prepare_t6(Plan* p);
 mdh_status launch_t6(const Plan& p, const void* const* in, void* const* out, void* ws, cudaStream_t st);
 void release_t4(Plan* p);
 
+// measured instruction-throughput peaks (peaks.cu; diagnostics)
+mdh_status measure_peaks(int device, double* ffma_tflops, double* alu_tops, double* issue_tops);
+
 // ordered ⊗-fold of S partial output sets (K-combine)
 mdh_status launch_combine(const Plan& p, const void* const* partials, int S, void* const* out,
                           cudaStream_t st);

@@ -102,6 +102,9 @@ def lib():
             L.mdh_last_launch_count.restype = ctypes.c_int32
             L.mdh_stencil_sweeps.argtypes = [P, P, P, ctypes.c_int32, ctypes.POINTER(Halo), P, S, P,
                                              ctypes.POINTER(ctypes.c_int32)]
+            D = ctypes.POINTER(ctypes.c_double)
+            L.mdh_measure_peaks.argtypes = [ctypes.c_int32, D, D, D]
+            L.mdh_measure_peaks.restype = ctypes.c_int
             L.mdh_debug_t4_trace.argtypes = [P, ctypes.c_int64]
             L.mdh_debug_t4_trace.restype = ctypes.c_int64
             for name in ("mdh_plan", "mdh_plan_workspace_size", "mdh_plan_local_shape", "mdh_plan_describe",
@@ -347,6 +350,13 @@ class Comm:
         if self.handle:
             lib().mdh_comm_destroy(self.handle)
             self.handle = None
+
+
+def measure_peaks(device: int = 0) -> dict:
+    """Measured FFMA / ALU-pipe / issue throughput of `device` (mdh_measure_peaks)."""
+    f, a, i = ctypes.c_double(), ctypes.c_double(), ctypes.c_double()
+    _check(lib().mdh_measure_peaks(int(device), ctypes.byref(f), ctypes.byref(a), ctypes.byref(i)))
+    return {"ffma_tflops": f.value, "alu_tops": a.value, "issue_tops": i.value}
 
 
 def abi_version() -> int:
