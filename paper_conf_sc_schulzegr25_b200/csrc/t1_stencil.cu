@@ -7,7 +7,11 @@
 // planes a stencil re-reads (z±1, y±1, x±1) are served from L1/L2 and every input
 // element comes from HBM about once (A2); f = Σ_a w_a·x_a (reading C-16) in fp32
 // with FMA (reading C-13).  HBM-bound: ≈8.05 B per output point for Jacobi3D.
+#include <cuda.h>
+#include <cudaTypedefs.h>
+
 #include <algorithm>
+#include <mutex>
 #include <type_traits>
 #include <vector>
 
@@ -207,6 +211,146 @@ __global__ void __launch_bounds__(128) t1_j3d7_kernel(const __grid_constant__ J7
     pc += P.Lz;
     po += P.oLz;
   }
+}
+
+// ---- TMA-staged 7-point cross (tile knob stages = ring depth ≥ 3) --------------------
+// A CTA owns a 128 × 32 (x × y) output tile and marches z over a z-chunk.  A producer warp
+// streams the input planes the chunk needs — a 132 × 34 box per plane, one
+// cp.async.bulk.tensor.3d each — into a ring of `stages` shared-memory planes (mbarrier
+// complete_tx), so several planes per CTA are in flight without holding registers; eight
+// compute warps read each output plane's 7 taps from the three resident input planes and
+// free the oldest plane as they finish.  The box starts one column left of the tile's first
+// centre (TMA box coordinates must be non-negative on this part: a negative start faults),
+// so a lane's row segment (left, 4 centres, right) is one aligned LDS.128 + LDS.64 and the
+// other taps an LDS.128 + LDS.32 each.  Box elements past the tensor end are zero-filled by
+// the TMA unit and never stored.
+constexpr int J7T_TX = 128, J7T_TY = 32, J7T_BX = 132, J7T_BY = J7T_TY + 2;
+constexpr int J7T_PLANE = J7T_BX * J7T_BY * 4;       // 9792 bytes loaded per plane
+constexpr int J7T_SLOT = (J7T_PLANE + 127) / 128 * 128;   // ring slot (TMA destinations 128-byte aligned)
+constexpr int J7T_THREADS = 288;                     // 8 compute warps + 1 producer warp
+constexpr int J7T_MAXS = 8;
+
+__device__ __forceinline__ void j7t_mbar_wait(uint32_t bar, uint32_t parity) {
+  asm volatile(
+      "{\n\t.reg .pred p;\n\t"
+      "WAIT_%=:\n\t"
+      "mbarrier.try_wait.parity.shared::cta.b64 p, [%0], %1;\n\t"
+      "@!p bra WAIT_%=;\n\t}" ::"r"(bar),
+      "r"(parity)
+      : "memory");
+}
+
+template <int VEC_OUT>
+__global__ void __launch_bounds__(J7T_THREADS) t1_j3d7_tma_kernel(const __grid_constant__ CUtensorMap map,
+                                                                  const __grid_constant__ J7Params P,
+                                                                  int stages, int cx, int cy, int cz, int ny) {
+  asm volatile("griddepcontrol.wait;" ::: "memory");
+  asm volatile("griddepcontrol.launch_dependents;" ::: "memory");
+  extern __shared__ __align__(1024) uint8_t j7t_raw[];
+  float* sm = (float*)(j7t_raw + ((1024u - ((uint32_t)__cvta_generic_to_shared(j7t_raw) & 1023u)) & 1023u));
+  __shared__ __align__(8) uint64_t bar_full[J7T_MAXS], bar_empty[J7T_MAXS];
+  const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
+  const int xb = blockIdx.x * J7T_TX, yb = blockIdx.y * J7T_TY;
+  const int z0 = blockIdx.z * P.zchunk, z1 = min(P.Z, z0 + P.zchunk);
+  const int nplanes = z1 - z0 + 2;                   // input planes z0 .. z1+1
+  const uint32_t sfull = (uint32_t)__cvta_generic_to_shared(bar_full);
+  const uint32_t sempty = (uint32_t)__cvta_generic_to_shared(bar_empty);
+  if (tid == 0) {
+    for (int s = 0; s < stages; ++s) {
+      asm volatile("mbarrier.init.shared::cta.b64 [%0], 1;" ::"r"(sfull + 8 * s));
+      asm volatile("mbarrier.init.shared::cta.b64 [%0], 256;" ::"r"(sempty + 8 * s));
+    }
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+  }
+  __syncthreads();
+  if (warp == 8) {
+    // ---- producer: plane j into slot j % stages (waits for the consumers to free it)
+    if (lane == 0) {
+      const uint32_t base = (uint32_t)__cvta_generic_to_shared(sm);
+      for (int j = 0; j < nplanes; ++j) {
+        const int s = j % stages;
+        if (j >= stages) j7t_mbar_wait(sempty + 8 * s, ((j / stages) - 1) & 1);
+        asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(sfull + 8 * s), "r"(J7T_PLANE)
+                     : "memory");
+        // the input viewed as 2-D rows [nz·ny][nx]: the box's 18 rows are rows yb+cy-1 … of
+        // plane z (rows past the plane end belong to the next plane — never stored)
+        asm volatile(
+            "cp.async.bulk.tensor.2d.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1, {%3, %4}], [%2];"
+            ::"r"(base + s * J7T_SLOT), "l"((uint64_t)&map), "r"(sfull + 8 * s), "r"(xb + cx - 1),
+            "r"((z0 + j + cz - 1) * ny + yb + cy - 1)
+            : "memory");
+      }
+    }
+  } else {
+  // ---- compute: warp w owns tile rows w, w + 8, …, lane l the outputs x = xb + 4l … +3
+  const int x = xb + 4 * lane;
+  const int nx = min(4, P.X - x);                    // valid outputs of this lane (≤ 0: none)
+  j7t_mbar_wait(sfull, 0);
+  j7t_mbar_wait(sfull + 8 * (1 % stages), (1 / stages) & 1);
+  for (int z = z0; z < z1; ++z) {
+    const int j = z - z0;
+    j7t_mbar_wait(sfull + 8 * ((j + 2) % stages), ((j + 2) / stages) & 1);
+    const float* pm = sm + (size_t)(j % stages) * (J7T_SLOT / 4);
+    const float* p0 = sm + (size_t)((j + 1) % stages) * (J7T_SLOT / 4);
+    const float* pp = sm + (size_t)((j + 2) % stages) * (J7T_SLOT / 4);
+#pragma unroll
+    for (int h = 0; h < J7T_TY / 8; ++h) {
+      const int ty = warp + 8 * h, y = yb + ty;
+      const int c = (ty + 1) * J7T_BX + 4 * lane;        // the left neighbour of output x in the box
+      const float4 ra = *reinterpret_cast<const float4*>(p0 + c);
+      const float2 rb = *reinterpret_cast<const float2*>(p0 + c + 4);
+      const float4 yma = *reinterpret_cast<const float4*>(p0 + c - J7T_BX);
+      const float4 ypa = *reinterpret_cast<const float4*>(p0 + c + J7T_BX);
+      const float4 zma = *reinterpret_cast<const float4*>(pm + c);
+      const float4 zpa = *reinterpret_cast<const float4*>(pp + c);
+      const float rr[6] = {ra.x, ra.y, ra.z, ra.w, rb.x, rb.y};
+      const float ymv[4] = {yma.y, yma.z, yma.w, p0[c - J7T_BX + 4]}, ypv[4] = {ypa.y, ypa.z, ypa.w, p0[c + J7T_BX + 4]};
+      const float zmv[4] = {zma.y, zma.z, zma.w, pm[c + 4]}, zpv[4] = {zpa.y, zpa.z, zpa.w, pp[c + 4]};
+      float o[4];
+#pragma unroll
+      for (int k = 0; k < 4; ++k) {
+        float acc = P.wc * rr[k + 1];
+        acc = fmaf(P.wxm, rr[k], acc);
+        acc = fmaf(P.wxp, rr[k + 2], acc);
+        acc = fmaf(P.wym, ymv[k], acc);
+        acc = fmaf(P.wyp, ypv[k], acc);
+        acc = fmaf(P.wzm, zmv[k], acc);
+        acc = fmaf(P.wzp, zpv[k], acc);
+        o[k] = acc;
+      }
+      if (y < P.Y && nx > 0) {
+        float* po = P.v + P.ob + x + (int64_t)y * P.oLy + (int64_t)z * P.oLz;
+        if (VEC_OUT == 1 && nx == 4) {
+          __stcs(reinterpret_cast<float2*>(po), make_float2(o[0], o[1]));
+          __stcs(reinterpret_cast<float2*>(po + 2), make_float2(o[2], o[3]));
+        } else if (VEC_OUT == 2 && nx == 4) {
+          __stcs(po, o[0]);
+          __stcs(reinterpret_cast<float2*>(po + 1), make_float2(o[1], o[2]));
+          __stcs(po + 3, o[3]);
+        } else {
+#pragma unroll
+          for (int k = 0; k < 4; ++k)
+            if (k < nx) po[k] = o[k];
+        }
+        if (z == 0 && P.hlo) {
+          float* q = P.hlo + P.hbase + x + (int64_t)y * P.oLy;
+#pragma unroll
+          for (int k = 0; k < 4; ++k)
+            if (k < nx) q[k] = o[k];
+        }
+        if (z == P.Z - 1 && P.hhi) {
+          float* q = P.hhi + P.hbase + x + (int64_t)y * P.oLy;
+#pragma unroll
+          for (int k = 0; k < 4; ++k)
+            if (k < nx) q[k] = o[k];
+        }
+      }
+    }
+    // input plane j is not needed by later output planes: free its slot
+    asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(sempty + 8 * (j % stages)) : "memory");
+  }
+  }
+  __syncthreads();
 }
 
 // ---- dense 2-D box stencil (H×W window, e.g. Gaussian_2D 5×5, Fig 3) -------
@@ -419,7 +563,11 @@ mdh_status prepare_t1(Plan* p) {
   if (detect_j3d7(p)) {
     p->ws_kernel = 0;
     p->t4_variant = 0;
-    p->why += " [7-point cross register-queue kernel]";
+    const Buf& B = p->in[0];
+    const int64_t Ly = B.acc[p->auxi[3]].L[p->auxi[1]], Lz = B.acc[p->auxi[3]].L[p->auxi[0]];
+    const bool tma = p->tiles.stages >= 3 && B.rank == 3 && B.shape[2] == Ly && B.shape[1] * B.shape[2] == Lz &&
+                     Ly % 4 == 0 && Lz % 4 == 0;
+    p->why += tma ? " [7-point cross, tma-staged plane ring]" : " [7-point cross register-queue kernel]";
     return MDH_OK;
   }
   if (detect_box2d(p)) {
@@ -486,6 +634,61 @@ static mdh_status launch_j3d7(const Plan& p, const void* const* in, void* const*
   // Measured on 512³ (zchunk 8, 3 interleaved reps on one box): none 206.8 µs, 128 B 206.8,
   // 256 B 204.8 (5212 GB/s; 8 sweeps 1.740 -> 1.732 ms); the z+1 row loaded one step ahead
   // (software pipeline along z, +8 registers) 206.9, with the 256 B hint 206.8 — dropped
+  // TMA-staged variant (tile knob stages = ring depth ≥ 3): the input must be a row-major
+  // [nz][ny][nx] buffer (x stride 1, Ly = nx, Lz = ny·nx) with 16-byte aligned rows and planes
+  const Buf& Bin = p.in[0];
+  const int st_ring = std::min(p.tiles.stages, J7T_MAXS);
+  if (st_ring >= 3 && Bin.rank == 3 && Bin.shape[2] == P.Ly && Bin.shape[1] * Bin.shape[2] == P.Lz && P.Ly % 4 == 0 &&
+      P.Lz % 4 == 0 && ((uintptr_t)P.u % 16) == 0 && P.oLy > 0) {
+    static PFN_cuTensorMapEncodeTiled_v12000 enc = nullptr;
+    static std::once_flag once;
+    std::call_once(once, [] {
+      void* f = nullptr;
+      cudaDriverEntryPointQueryResult q;
+      if (cudaGetDriverEntryPoint("cuTensorMapEncodeTiled", &f, cudaEnableDefault, &q) == cudaSuccess &&
+          q == cudaDriverEntryPointSuccess)
+        enc = (PFN_cuTensorMapEncodeTiled_v12000)f;
+    });
+    if (!enc) { set_error("cuTensorMapEncodeTiled unavailable"); return MDH_ERR_CUDA; }
+    CUtensorMap map;
+    cuuint64_t dims[2] = {(cuuint64_t)Bin.shape[2], (cuuint64_t)(Bin.shape[1] * Bin.shape[0])};
+    cuuint64_t strides[1] = {(cuuint64_t)P.Ly * 4};
+    cuuint32_t box[2] = {J7T_BX, J7T_BY};
+    cuuint32_t estr[2] = {1, 1};
+    CUresult r = enc(&map, CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 2, (void*)P.u, dims, strides, box, estr,
+                     CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_NONE, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
+                     CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+    if (r != CUDA_SUCCESS) { set_error("cuTensorMapEncodeTiled (stencil input) failed (%d)", (int)r); return MDH_ERR_CUDA; }
+    // input coordinate of the centre access at the iteration origin
+    const int cz = (int)(P.bc / P.Lz), cy = (int)((P.bc % P.Lz) / P.Ly), cx = (int)(P.bc % P.Ly);
+    const size_t smem = (size_t)st_ring * J7T_SLOT + 1024;
+    void (*tk)(CUtensorMap, J7Params, int, int, int, int, int) =
+        vout ? t1_j3d7_tma_kernel<1> : (vodd ? t1_j3d7_tma_kernel<2> : t1_j3d7_tma_kernel<0>);
+    static std::once_flag attr_once;
+    static cudaError_t attr_err = cudaSuccess;
+    std::call_once(attr_once, [] {
+      for (auto k : {t1_j3d7_tma_kernel<0>, t1_j3d7_tma_kernel<1>, t1_j3d7_tma_kernel<2>}) {
+        const cudaError_t e = cudaFuncSetAttribute((const void*)k, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                                   J7T_MAXS * J7T_SLOT + 1024);
+        if (e != cudaSuccess) attr_err = e;
+      }
+    });
+    MDH_CUDA(attr_err);
+    dim3 tgrid((unsigned)((P.X + J7T_TX - 1) / J7T_TX), (unsigned)((P.Y + J7T_TY - 1) / J7T_TY),
+               (unsigned)((P.Z + zc - 1) / zc));
+    cudaLaunchConfig_t cfg = {};
+    cfg.gridDim = tgrid;
+    cfg.blockDim = dim3(J7T_THREADS);
+    cfg.dynamicSmemBytes = smem;
+    cfg.stream = st;
+    cudaLaunchAttribute attr[1];
+    attr[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+    attr[0].val.programmaticStreamSerializationAllowed = 1;
+    cfg.attrs = attr;
+    cfg.numAttrs = pdl ? 1 : 0;
+    MDH_CUDA(cudaLaunchKernelEx(&cfg, tk, map, P, st_ring, cx, cy, cz, (int)Bin.shape[1]));
+    return post_launch("t1_j3d7_tma_kernel");
+  }
   const int pf = p.tiles.l2pf;
   void (*kern)(J7Params) = nullptr;
 #define J7(VI, VO)                                              \

@@ -236,6 +236,27 @@ def test_mcc_fp32(cfg):
     assert_close_full(spec, x, got, 1e-4, kind="scale")
 
 
+@pytest.mark.parametrize("zyx", [(5, 7, 12), (66, 130, 260), (34, 19, 136), (64, 64, 64), (512, 512, 512)])
+@pytest.mark.parametrize("tile", ["stages=3,zchunk=8", "stages=6,zchunk=16"])
+def test_jacobi3d_tma_staged(zyx, tile):
+    """The TMA-staged 7-point kernel (tile knob stages ≥ 3: input planes streamed into a
+    shared-memory ring by cp.async.bulk.tensor; rows of a multiple of 4 floats, the
+    kernel's eligibility): ragged x/y/z tiles, tiny grids, full
+    size (sampled), against the oracle (scale-normalised 1e-4) and bit-identical to the
+    register-queue kernel (same per-point arithmetic)."""
+    Z, Y, X = zyx
+    spec = S.jacobi3d(Z, Y, X)
+    x = G.jacobi3d_inputs(Z, Y, X)
+    got, p = run_gpu(spec, x, force_tile=tile)
+    assert "tma" in p.describe()["why"], p.describe()["why"]
+    ref, _ = run_gpu(spec, x, force_tile="stages=0")
+    assert np.array_equal(got[0], ref[0])
+    if Z * Y * X <= 66 * 130 * 258:
+        assert_close_full(spec, x, got, 1e-4, kind="scale")
+    else:
+        assert_close_points(spec, x, got, 1e-4, n=20000, kind="scale")
+
+
 # ----------------------------------------------------------------- T5: PRL
 @pytest.mark.parametrize("op", ["PW_PRL_ARGMAX", "PW_PRL_PAPER"])
 def test_prl_tiny_golden(op):

@@ -108,6 +108,12 @@ def main():
             for kv in best[1].split(","):
                 k, v = kv.split("=")
                 tiles[k] = int(v)
+        else:
+            # the default won: record the knobs it resolved to (a table entry of {} would
+            # fall back to the template defaults, not to the nearest bucket it was timed with)
+            knobs = {"T1_stencil": ("zchunk", "l2pf"), "T2_reduce": ("split",), "T4_tcgen05_contraction": ("bn", "split"),
+                     "T5_prl_pairwise": ("split",), "T3_simt_contraction": ("split",)}.get(d["template"], ())
+            tiles = {k: int(d["tiles"][k]) for k in knobs if k in d["tiles"]}
         key = (d["template"], dtype, tuple(bucket))
         entries[key] = {"template": d["template"], "dtype": dtype, "bucket": bucket, "tiles": tiles,
                         "workload": name, "median_us": round(best[0] * 1e6, 2),
