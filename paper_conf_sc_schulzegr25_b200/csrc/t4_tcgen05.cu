@@ -993,13 +993,19 @@ __device__ __forceinline__ void mbar_arrive_cluster(uint32_t bar_cluster) {
 // next tile's first MMAs into half h wait only for tempty[h].  Per k-block a CTA loads its
 // A half once for twice the MMA work (A 16 + B 32 KB per 8.4 MFLOP instead of 16 + 16 per
 // 4.2): A — the im2col operand of a convolution — is requested half as often.
-template <bool OUT_ROWMAJOR, int CL, int NW = 256>
+// WST (wide tiles only): ring stages — 3 with double-buffered epilogue staging, or 4 with
+// single-buffered staging (4 × 48 KB + 32 KB fits the 227 KB budget; tile knob stages=4:
+// MCC conv5_1 +1-3 %, MatMul 4096³ / 8192³ -2 / -3 %: the single staging buffer slows the
+// whole-tile epilogues)
+template <bool OUT_ROWMAJOR, int CL, int NW = 256, int WST = S2W>
 __global__ void __cluster_dims__(CL, 1, 1) __launch_bounds__(THREADS, 1)
     gemm2_kernel(const __grid_constant__ CUtensorMap mapA, const __grid_constant__ CUtensorMap mapB,
                  const __grid_constant__ CUtensorMap mapC, const __grid_constant__ Params P) {
   extern __shared__ __align__(1024) uint8_t smem_raw[];
   constexpr int NH = NW / 256;                   // N=256 MMAs per k-step
-  constexpr int NS = NW == 512 ? S2W : S2;       // ring stages
+  constexpr int NS = NW == 512 ? WST : S2;       // ring stages
+  constexpr int EPB = (NW == 512 && WST == 4) ? 1 : 2;   // epilogue staging buffers per warp
+  static_assert(NW != 512 || WST * (A2_BYTES + 2 * B2_BYTES) + 2048 + EPB * 8 * 4096 <= 232448, "smem budget");
   constexpr int BSTG = NH * B2_BYTES;            // this CTA's B bytes per stage
   uint8_t* smem = (uint8_t*)(((uintptr_t)smem_raw + 1023) & ~(uintptr_t)1023);
   uint8_t* sA = smem;
@@ -1171,7 +1177,7 @@ __global__ void __cluster_dims__(CL, 1, 1) __launch_bounds__(THREADS, 1)
     const int row = quad * 32 + lane;
     const int ew = rank * 8 + (warp - 2);          // this warp's slot in a stream-K partial
     // (1024-byte aligned: the TMA 128B swizzle pattern is a function of the address bits)
-    const uint32_t stg0 = smem_u32(smem + NS * (A2_BYTES + BSTG) + 1024) + (warp - 2) * 8192;
+    const uint32_t stg0 = smem_u32(smem + NS * (A2_BYTES + BSTG) + 1024) + (warp - 2) * (EPB * 4096);
     int sbuf = 0;                                  // staging buffer of the next TMA store
     const uint32_t tempty_leader = map_to_rank(tempty0, 2 * pp);
     int it = 0;
@@ -1242,7 +1248,10 @@ __global__ void __cluster_dims__(CL, 1, 1) __launch_bounds__(THREADS, 1)
           // 32×32 box (rows / columns beyond M / N are clipped by the TMA unit); two staging
           // buffers per warp, so a buffer is rewritten only after its previous store read it
           const uint32_t stg = stg0 + sbuf * 4096;
-          if (lane == 0) asm volatile("cp.async.bulk.wait_group.read 1;" ::: "memory");
+          if (lane == 0) {
+            if (EPB == 2) asm volatile("cp.async.bulk.wait_group.read 1;" ::: "memory");
+            else asm volatile("cp.async.bulk.wait_group.read 0;" ::: "memory");
+          }
           __syncwarp();
 #pragma unroll
           for (int j = 0; j < 8; ++j)
@@ -1255,7 +1264,7 @@ __global__ void __cluster_dims__(CL, 1, 1) __launch_bounds__(THREADS, 1)
             tma_store_2d(&mapC, stg, (int)nb, (int)(m - row + quad * 32));
             asm volatile("cp.async.bulk.commit_group;" ::: "memory");
           }
-          sbuf ^= 1;
+          sbuf ^= EPB - 1;
         } else if (OUT_ROWMAJOR && mok && nb + 32 <= P.N && ((crow + nb) & 3) == 0) {
           float4* dst = reinterpret_cast<float4*>(P.C + crow + nb);
 #pragma unroll
@@ -1546,6 +1555,7 @@ struct T4State {
   int cg = 1;      // 1: one SM per 128×256 tile; 2: SM pair per 256×256 tile
   int cl = 2;      // 2-SM kernel: CTAs per cluster (4: two pairs share B by multicast)
   int nw = 256;    // 2-SM kernel: N extent of a pair tile (512: two MMAs per k-step)
+  int wst = 3;     // wide 2-SM ring stages (4: single-buffered epilogue staging; tile knob stages=4)
   bool sk_ok = false;   // 2-SM kernel: stream-K workspace reserved
   bool ag = false; // A staged by the kernel's gather warps (no A tensor map, no pre-pass)
   bool ic = false;  // A through a TMA im2col map
@@ -1690,6 +1700,7 @@ mdh_status prepare_t4(Plan* p) {
   if (prepare_t4_conv(p)) return MDH_OK;           // small-K direct variant (t4_conv.cu)
   const Contraction& c = p->con;
   T4State* s = new T4State();
+  s->wst = p->tiles.stages == 4 ? 4 : 3;
   size_t ws = 0;
   std::string w2;
   const t4::Layout2D a_direct = t4::operand_layout(*p, c.md, c.nm, c.M, p->in[c.a_buf].acc[0], &w2, "A");
@@ -1951,7 +1962,7 @@ mdh_status prepare_t4(Plan* p) {
   p->tiles.bm = s->cg == 2 ? 256 : t4::BM;
   p->tiles.bn = s->epi == 3 ? P.bn : (s->cg == 2 ? s->nw : t4::BN);
   p->tiles.bk = t4::BK;
-  p->tiles.stages = s->cg == 2 ? t4::S2 : (s->epi == 3 ? 2 : t4::STAGES);
+  p->tiles.stages = s->cg == 2 ? (s->nw == 512 ? s->wst : t4::S2) : (s->epi == 3 ? 2 : t4::STAGES);
   p->tiles.cluster = s->cg == 2 ? s->cl : 1;
   return MDH_OK;
 }
@@ -2165,9 +2176,9 @@ mdh_status launch_t4(const Plan& p, const void* const* in, void* const* out, voi
                                            (int)(t4::SMEM_LIMIT - t4::BN * sizeof(int64_t)));
       if (e != cudaSuccess) attr_err = e;
     }
-    const void* k2[5] = {(const void*)t4::gemm2_kernel<true, 2>, (const void*)t4::gemm2_kernel<false, 2>,
+    const void* k2[6] = {(const void*)t4::gemm2_kernel<true, 2>, (const void*)t4::gemm2_kernel<false, 2>,
                          (const void*)t4::gemm2_kernel<true, 4>, (const void*)t4::gemm2_kernel<false, 4>,
-                         (const void*)t4::gemm2_kernel<true, 2, 512>};
+                         (const void*)t4::gemm2_kernel<true, 2, 512>, (const void*)t4::gemm2_kernel<true, 2, 512, 4>};
     for (const void* k : k2) {
       cudaError_t e = cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, t4::SMEM2_BYTES);
       if (e != cudaSuccess) attr_err = e;
@@ -2256,7 +2267,9 @@ mdh_status launch_t4(const Plan& p, const void* const* in, void* const* out, voi
                       CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
       if (r != CUDA_SUCCESS) { set_error("cuTensorMapEncodeTiled (C store map) failed (%d)", (int)r); return MDH_ERR_CUDA; }
     }
-    if (s->nw == 512) t4::gemm2_kernel<true, 2, 512><<<grid2, t4::THREADS, t4::SMEM2_BYTES, st>>>(ma, mb, mc, P);
+    if (s->nw == 512 && s->wst == 4)
+      t4::gemm2_kernel<true, 2, 512, 4><<<grid2, t4::THREADS, t4::SMEM2_BYTES, st>>>(ma, mb, mc, P);
+    else if (s->nw == 512) t4::gemm2_kernel<true, 2, 512><<<grid2, t4::THREADS, t4::SMEM2_BYTES, st>>>(ma, mb, mc, P);
     else if (CL == 4) t4::gemm2_kernel<true, 4><<<grid2, t4::THREADS, t4::SMEM2_BYTES, st>>>(ma, mb, mc, P);
     else t4::gemm2_kernel<true, 2><<<grid2, t4::THREADS, t4::SMEM2_BYTES, st>>>(ma, mb, mc, P);
     return post_launch("t4_gemm2_kernel");

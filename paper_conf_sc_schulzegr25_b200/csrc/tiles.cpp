@@ -162,7 +162,8 @@ void lookup_tiles(Plan* p, const char* table_path, const char* force) {
   Tiles t;
   // template defaults
   if (p->tmpl == T1_STENCIL) { t.zchunk = 32; t.stages = 0; }   // stages ≥ 3: TMA-staged 7-point kernel
-  if (p->tmpl == T4_TC) { t.bm = 128; t.bn = 0; t.bk = 64; t.stages = 4; t.cluster = 0; }   // bn, cluster 0 = auto
+  // T4: bn, cluster, stages 0 = auto (stages = 4 selects the 4-stage wide 2-SM ring)
+  if (p->tmpl == T4_TC) { t.bm = 128; t.bn = 0; t.bk = 64; t.stages = 0; t.cluster = 0; }
   // T5: 4 new records per thread, registers for 3 CTAs per SM, DB loop unrolled ×4 (t5_prl.cu)
   if (p->tmpl == T5_PRL) { t.vec = 4; t.stages = 3; t.bk = 4; }
   std::string text;
