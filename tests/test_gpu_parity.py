@@ -163,6 +163,24 @@ def test_copy_identity():
     assert np.array_equal(got[0], x[0])
 
 
+@pytest.mark.parametrize("dt", ["u32", "i64"])
+@pytest.mark.parametrize("op", ["PW_ADD", "PW_MAX", "PW_MIN"])
+def test_dot_u32_i64_wrap_and_order(dt, op):
+    """uint32 (mod 2^32, unsigned order) and int64 (mod 2^64) reductions on T2, bit-exact
+    against the oracle's u32 / i64 kinds (pinned against Python integers on the CPU)."""
+    g = np.random.Generator(np.random.PCG64(62))
+    n = 100003
+    if dt == "u32":
+        a = g.integers(0, 2 ** 32, n, dtype=np.uint64).astype(np.uint32)
+        b = g.integers(0, 2 ** 32, n, dtype=np.uint64).astype(np.uint32)
+    else:
+        a = g.integers(-2 ** 40, 2 ** 40, n).astype(np.int64)
+        b = g.integers(-2 ** 30, 2 ** 30, n).astype(np.int64)
+    spec = S.dot(n, dt, op)
+    got, _ = run_gpu(spec, [a, b])
+    assert_close_full(spec, [a, b], got, 0, kind="exact")
+
+
 # ----------------------------------------------------------------- T3: SIMT contraction
 @pytest.mark.parametrize("mnk", [(1, 1, 1), (3, 5, 7), (127, 129, 65), (128, 256, 64), (300, 200, 1000)])
 def test_matmul_fp32(mnk):

@@ -79,6 +79,32 @@ def test_dot_maxmin(op, fn, dt):
 
 
 # --------------------------------------------------------------- MatMul (C2)
+def test_u32_and_i64_wrap_branches():
+    """The oracle's uint32 (mod 2^32, unsigned order) and int64 (mod 2^64) kinds against
+    Python's unbounded integers reduced by hand — independent of numpy's own wrapping."""
+    g = np.random.Generator(np.random.PCG64(61))
+    n = 3001
+    a = g.integers(0, 2 ** 32, n, dtype=np.uint64).astype(np.uint32)
+    b = g.integers(0, 2 ** 32, n, dtype=np.uint64).astype(np.uint32)
+    exact = sum(int(x) * int(y) for x, y in zip(a.tolist(), b.tolist()))
+    got = int(oracle.evaluate(S.dot(n, "u32"), [a, b])[0][0])
+    assert got == exact % 2 ** 32
+    # unsigned order: products ≥ 2^31 must win a max / lose a min as unsigned values
+    prods = [(int(x) * int(y)) % 2 ** 32 for x, y in zip(a.tolist(), b.tolist())]
+    assert int(oracle.evaluate(S.dot(n, "u32", "PW_MAX"), [a, b])[0][0]) == max(prods)
+    assert int(oracle.evaluate(S.dot(n, "u32", "PW_MIN"), [a, b])[0][0]) == min(prods)
+    # int64: products of ~2^40 × ~2^30 overflow 2^63; the sum wraps mod 2^64 (two's complement)
+    x = (g.integers(-2 ** 40, 2 ** 40, n)).astype(np.int64)
+    y = (g.integers(-2 ** 30, 2 ** 30, n)).astype(np.int64)
+    exact = sum(int(p) * int(q) for p, q in zip(x.tolist(), y.tolist())) % 2 ** 64
+    exact = exact - 2 ** 64 if exact >= 2 ** 63 else exact
+    assert int(oracle.evaluate(S.dot(n, "i64"), [x, y])[0][0]) == exact
+    prods64 = [int(p) * int(q) for p, q in zip(x.tolist(), y.tolist())]
+    wrap64 = [((v + 2 ** 63) % 2 ** 64) - 2 ** 63 for v in prods64]
+    assert int(oracle.evaluate(S.dot(n, "i64", "PW_MAX"), [x, y])[0][0]) == max(wrap64)
+    assert int(oracle.evaluate(S.dot(n, "i64", "PW_MIN"), [x, y])[0][0]) == min(wrap64)
+
+
 def test_matmul_identity_and_ones():
     M = K = 48
     N = 40
