@@ -2,8 +2,11 @@
 //
 // Template parameters come from a table produced by a MEASURED sweep on B200
 // (tools/sweep_tiles.py → tiles/b200.json; the ATF auto-tuning of P:497-501 is prior
-// art, replaced by this sweep).  Key: (template, dtype, shape bucket), the bucket being
-// the log2-rounded extents of (Ncc, Nred) or (M, N, K) of THIS rank's sub-problem.
+// art, replaced by this sweep).  Key: (template, dtype, f, ⊗-class, shape bucket), the
+// bucket being the log2-rounded extents of (Ncc, Nred) or (M, N, K) of THIS rank's
+// sub-problem; f ("MUL", "STENCIL", "PRL_COMPARE", "IDENTITY") and the ⊗-class (the
+// common pw operator: "PW_ADD", …, "PS_ADD", or "CC") must match when an entry records
+// them (entries without them match any f / ⊗).
 // Lookup: exact bucket, else the nearest bucket of the same template and dtype by
 // log-distance, else the template's defaults.  Overrides: the plan option force_tile or
 // $MDH_FORCE_TILE ("split=4,zchunk=16,…").  Table: the plan option, $MDH_TILE_TABLE, or
@@ -130,6 +133,28 @@ void shape_key(const Plan& p, double key[3]) {
   }
 }
 
+const char* fn_name(mdh_fn f) {
+  switch (f) {
+    case MDH_F_MUL: return "MUL";
+    case MDH_F_STENCIL: return "STENCIL";
+    case MDH_F_PRL_COMPARE: return "PRL_COMPARE";
+    case MDH_F_IDENTITY: return "IDENTITY";
+  }
+  return "?";
+}
+
+const char* op_class(const Plan& p) {
+  if (p.nps > 0) return "PS_ADD";
+  switch (p.redop) {
+    case MDH_PW_ADD: return "PW_ADD";
+    case MDH_PW_MAX: return "PW_MAX";
+    case MDH_PW_MIN: return "PW_MIN";
+    case MDH_PW_PRL_ARGMAX: return "PW_PRL_ARGMAX";
+    case MDH_PW_PRL_PAPER: return "PW_PRL_PAPER";
+    default: return "CC";
+  }
+}
+
 void apply(Tiles* t, const std::string& k, double v) {
   int iv = (int)v;
   if (k == "threads") t->threads = iv;
@@ -186,6 +211,9 @@ void lookup_tiles(Plan* p, const char* table_path, const char* force) {
       const J* ed = e.get("dtype");
       const J* eb = e.get("bucket");
       if (!et || !ed || !eb || et->str != tname || ed->str != dname || eb->t != J::ARR) continue;
+      const J* ef = e.get("f");
+      const J* eo = e.get("op");
+      if ((ef && ef->str != fn_name(p->f)) || (eo && eo->str != op_class(*p))) continue;
       double d = 0;
       for (size_t i = 0; i < eb->arr.size() && i < 3; ++i) d += std::fabs(eb->arr[i].num - key[i]);
       if (d < bestd) { bestd = d; best = &e; }

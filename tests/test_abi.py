@@ -154,6 +154,11 @@ def test_tile_override_and_table(mdh, tmp_path):
     assert d["tiles"]["split"] == 33 and d["tiles"]["source"].startswith("table")
     d = mdh.Plan(S.dot(1 << 22, "f32"), tile_table=str(t)).describe()   # nearest bucket
     assert d["tiles"]["split"] == 33
+    # the key includes f and the ⊗-class when an entry records them
+    t.write_text('{"entries": [{"template": "T2_reduce", "dtype": "f32", "f": "MUL", "op": "PW_MAX", '
+                 '"bucket": [0, 20], "tiles": {"split": 44}}]}')
+    assert mdh.Plan(S.dot(1 << 20, "f32", "PW_MAX"), tile_table=str(t)).describe()["tiles"]["split"] == 44
+    assert mdh.Plan(S.dot(1 << 20, "f32"), tile_table=str(t)).describe()["tiles"]["source"] == "default"
 
 
 def test_sweeps_argument_checks_on_host(mdh):

@@ -71,7 +71,7 @@ def main():
     dev = torch.device("cuda", 0)
     flush = bench.L2Flush(dev)
     table = json.load(open(a.out)) if os.path.exists(a.out) else {"entries": []}
-    entries = {(e["template"], e["dtype"], tuple(e["bucket"])): e for e in table.get("entries", [])}
+    entries = {(e["template"], e["dtype"], e.get("f"), e.get("op"), tuple(e["bucket"])): e for e in table.get("entries", [])}
     log = []
     for name, mk, cands in cases():
         if a.only and a.only not in name:
@@ -114,8 +114,10 @@ def main():
             knobs = {"T1_stencil": ("zchunk", "l2pf"), "T2_reduce": ("split",), "T4_tcgen05_contraction": ("bn", "split"),
                      "T5_prl_pairwise": ("split",), "T3_simt_contraction": ("split",)}.get(d["template"], ())
             tiles = {k: int(d["tiles"][k]) for k in knobs if k in d["tiles"]}
-        key = (d["template"], dtype, tuple(bucket))
-        entries[key] = {"template": d["template"], "dtype": dtype, "bucket": bucket, "tiles": tiles,
+        fname = spec["f"]
+        opcls = next((o for o in spec["ops"] if o == "PS_ADD"), None) or next((o for o in spec["ops"] if o != "CC"), "CC")
+        key = (d["template"], dtype, fname, opcls, tuple(bucket))
+        entries[key] = {"template": d["template"], "dtype": dtype, "f": fname, "op": opcls, "bucket": bucket, "tiles": tiles,
                         "workload": name, "median_us": round(best[0] * 1e6, 2),
                         "default_us": round(res[0][0] * 1e6, 2),
                         "sweep": {(r[1] or "default"): round(r[0] * 1e6, 2) for r in res}}
