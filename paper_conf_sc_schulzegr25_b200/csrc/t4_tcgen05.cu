@@ -101,6 +101,13 @@ struct Params {
   // k-blocks, cut into sk_pairs equal contiguous ranges, one per pair (0 = off)
   int sk_pairs;
   int64_t sk_w;
+  // column-unit stream (wide 2-SM kernel, vmode): the output is cut into 256-row strips and
+  // 128-column units (ups per strip, vunits in all); pair p owns units
+  // [p·vunits/npairs, (p+1)·vunits/npairs) — whole K, no partial sums — as tiles of ≤ 4
+  // units that never cross a strip, so the pairs' work differs by at most one unit
+  int vmode, ups;
+  int64_t vunits;
+  uint32_t idesc128;                // the N = 128 instruction descriptor (a tile's odd last unit)
   float* skpart;                    // one fp32 256×256 partial tile per pair (coalesced layout)
   unsigned* skflag;                 // 16 flags per pair (2 CTAs × 8 epilogue warps); zero at rest
   // diagnostics: per-unit timeline (MDH_T4_TRACE=1; 2-SM kernel), 4 u64 per unit:
@@ -871,22 +878,38 @@ __global__ void __launch_bounds__(AG ? THREADS + AG_THREADS : THREADS, 1)
 // adds the producers' partials p+1, p+2, … in k order before the store).  Producers run
 // first and finishers last, so a finisher finds its partials (nearly always) published;
 // all pairs are co-resident (persistent grid), so the flag waits cannot deadlock.
-struct SkWork { int t, kb0, kb1, role; };
+struct SkWork { int t, kb0, kb1, role, u0, nu; };   // u0 / nu: first column unit and units (vmode)
 struct SkIter {
-  int u, step, nfull, kb;
+  int u, step, nfull, kb, ups;
+  bool vmode;
   int64_t k, e;
   __device__ __forceinline__ SkIter(const Params& P, int pair, int npairs) {
     u = pair;
     step = npairs;
     nfull = P.nfull;
     kb = P.num_kb;
+    vmode = P.vmode != 0;
+    ups = P.ups;
     k = e = 0;
-    if (P.sk_pairs > 0 && pair < P.sk_pairs) {
+    if (vmode) {
+      k = (int64_t)pair * P.vunits / npairs;
+      e = (int64_t)(pair + 1) * P.vunits / npairs;
+    } else if (P.sk_pairs > 0 && pair < P.sk_pairs) {
       k = (int64_t)pair * P.sk_w / P.sk_pairs;
       e = (int64_t)(pair + 1) * P.sk_w / P.sk_pairs;
     }
   }
   __device__ __forceinline__ bool next(SkWork* w) {
+    w->u0 = 0;
+    w->nu = 0;
+    if (vmode) {                     // units k … e-1: strip k / ups, ≤ 4 units per tile
+      if (k >= e) return false;
+      const int strip = (int)(k / ups), cu = (int)(k % ups);
+      const int nu = (int)min((int64_t)4, min(e - k, (int64_t)(ups - cu)));
+      w->t = strip; w->kb0 = 0; w->kb1 = kb; w->role = 0; w->u0 = cu; w->nu = nu;
+      k += nu;
+      return true;
+    }
     if (u < nfull) {
       w->t = u; w->kb0 = 0; w->kb1 = kb; w->role = 0;
       u += step;
@@ -1059,11 +1082,18 @@ __global__ void __cluster_dims__(CL, 1, 1) __launch_bounds__(THREADS, 1)
       SkWork w;
       while (wi.next(&w)) {
         const int t = w.t, kb0 = w.kb0, kb1 = w.kb1;
-        const int m0 = ((t / P.tiles_n) * NPP + (int)pp) * 256 + (int)rank * 128, n0 = (t % P.tiles_n) * NW + (int)rank * 128;
+        const int m0 = P.vmode ? t * 256 + (int)rank * 128 : ((t / P.tiles_n) * NPP + (int)pp) * 256 + (int)rank * 128;
+        const int n0 = P.vmode ? 128 * w.u0 + (int)rank * 128 : (t % P.tiles_n) * NW + (int)rank * 128;
+        // vmode: MMA h covers units u0+2h, u0+2h+1 (N = 256, 128 columns per CTA) or only the
+        // tile's odd last unit (N = 128, 64 columns per CTA: one 64-column MN-major box)
+        const int vnh = (w.nu + 1) / 2;
+        const bool vodd = (w.nu & 1) != 0;
+        const uint32_t bbytes = !P.vmode ? (uint32_t)BSTG
+                                         : (uint32_t)(vnh * B2_BYTES - (vodd && P.b_mn_major ? B2_BYTES / 2 : 0));
         for (int kb = kb0; kb < kb1; ++kb) {
           mbar_wait(empty0 + 8 * stage, phase ^ 1);
           const uint32_t fb_leader = map_to_rank(full0 + 8 * stage, 2 * pp);
-          if (leader) mbar_expect_tx(full0 + 8 * stage, 2 * (A2_BYTES + BSTG));
+          if (leader) mbar_expect_tx(full0 + 8 * stage, 2 * (A2_BYTES + bbytes));
           else mbar_arrive_cluster(fb_leader);
           const uint32_t a_dst = smem_u32(sA + stage * A2_BYTES), b_dst = smem_u32(sB + stage * BSTG);
           const int k0 = krotate(P, kb, kb0, kb1, t / P.tiles_n) * BK;
@@ -1082,6 +1112,17 @@ __global__ void __cluster_dims__(CL, 1, 1) __launch_bounds__(THREADS, 1)
             const uint16_t mask = (uint16_t)((1u << rank) | (1u << (2 + rank)));
             if (P.b_mn_major) tma_load_2d_cg2_mc(b_dst + pp * 8192, &mapB, fb_leader, n0 + 64 * pp, k0, mask);
             else tma_load_2d_cg2_mc(b_dst + pp * 8192, &mapB, fb_leader, k0, n0 + 64 * pp, mask);
+          } else if (P.vmode) {
+            for (int h = 0; h < vnh; ++h) {
+              const bool half_unit = vodd && h == vnh - 1;     // N = 128: 64 columns per CTA
+              const int nb = half_unit ? 128 * (w.u0 + 2 * h) + (int)rank * 64 : n0 + 256 * h;
+              if (P.b_mn_major) {
+                tma_load_2d_cg2(b_dst + h * B2_BYTES, &mapB, fb_leader, nb, k0);
+                if (!half_unit) tma_load_2d_cg2(b_dst + h * B2_BYTES + 8192, &mapB, fb_leader, nb + 64, k0);
+              } else {
+                tma_load_2d_cg2(b_dst + h * B2_BYTES, &mapB, fb_leader, k0, nb);
+              }
+            }
           } else {
 #pragma unroll
             for (int h = 0; h < NH; ++h) {   // B piece h: columns 256h + 128·rank + [0, 128)
@@ -1132,8 +1173,11 @@ __global__ void __cluster_dims__(CL, 1, 1) __launch_bounds__(THREADS, 1)
             P.trace[8 * (pair_gid + u * nclusters * NPP) + 1] = gtimer();
           }
           const uint32_t a0 = smem_u32(sA + stage * A2_BYTES), b0 = smem_u32(sB + stage * BSTG);
+          const int mnh = P.vmode ? (w.nu + 1) / 2 : NH;
 #pragma unroll
           for (int h = 0; h < NH; ++h) {
+            if (h >= mnh) break;
+            const uint32_t idesc_h = (P.vmode && (w.nu & 1) && h == mnh - 1) ? P.idesc128 : P.idesc;
             if (NH > 1 && kb == kb0) {      // column half h of the accumulator drained?
               const long long ch = P.trace ? clock64() : 0;
               mbar_wait(tempty0 + 8 * h, (it & 1) ^ 1);
@@ -1146,7 +1190,7 @@ __global__ void __cluster_dims__(CL, 1, 1) __launch_bounds__(THREADS, 1)
               const uint64_t ad = P.a_mn_major ? sdesc(a0 + 2048 * k, 8192, 1024) : sdesc(a0 + 32 * k, 16, 1024);
               const uint32_t bh = b0 + h * B2_BYTES;
               const uint64_t bd = P.b_mn_major ? sdesc(bh + 2048 * k, 8192, 1024) : sdesc(bh + 32 * k, 16, 1024);
-              mma_bf16_cg2(d + 256 * h, ad, bd, P.idesc, (kb != kb0) || k != 0);
+              mma_bf16_cg2(d + 256 * h, ad, bd, idesc_h, (kb != kb0) || k != 0);
             }
           }
           if (CL == 4) mma_commit_cg2_mask(empty0 + 8 * stage, 0xF);
@@ -1186,8 +1230,11 @@ __global__ void __cluster_dims__(CL, 1, 1) __launch_bounds__(THREADS, 1)
     for (; wi.next(&w); ++it) {
       const int t = w.t;
       const int acc = NH == 1 ? it & 1 : 0;
-      const int64_t m = ((int64_t)(t / P.tiles_n) * NPP + pp) * 256 + rank * 128 + row;
-      const int64_t ntile = (int64_t)(t % P.tiles_n) * NW;
+      const int64_t m = P.vmode ? (int64_t)t * 256 + rank * 128 + row
+                                : ((int64_t)(t / P.tiles_n) * NPP + pp) * 256 + rank * 128 + row;
+      const int64_t ntile = P.vmode ? (int64_t)128 * w.u0 : (int64_t)(t % P.tiles_n) * NW;
+      // columns of this tile held by this warp group in MMA half h (vmode: a group may hold none)
+      auto group_has = [&](int h) { return !P.vmode || 2 * h + half < w.nu; };
       mbar_wait(tfull0 + 8 * acc, NH == 1 ? (it >> 1) & 1 : it & 1);
       tc_fence_after();
       const bool mok = m < P.M;
@@ -1279,6 +1326,14 @@ __global__ void __cluster_dims__(CL, 1, 1) __launch_bounds__(THREADS, 1)
       };
 #pragma unroll 1
       for (int h = 0; h < NH; ++h) {
+      if (!group_has(h)) {             // nothing of this half for this group: release it at once
+        if (NH > 1) {
+          tc_fence_before();
+          __syncwarp();
+          if (lane == 0) mbar_arrive_cluster(tempty_leader + 8 * h);
+        }
+        continue;
+      }
       const int64_t n0 = ntile + 256 * h + half * 128;
       const uint32_t tb = tmem + ((uint32_t)(quad * 32) << 16) + acc * BN + 256 * h + half * 128;
       // (a software-pipelined variant — TMEM load of chunk c+1 in flight while chunk c is
@@ -2246,7 +2301,19 @@ mdh_status launch_t4(const Plan& p, const void* const* in, void* const* out, voi
         P.skflag = (unsigned*)((char*)ws + s->tail_off + (size_t)t4::SK_MAX_PAIRS * (s->nw / 256) * 65536 * sizeof(float));
       }
     }
-    const int clusters = P.sk_pairs > 0 ? C : std::max(1, std::min(T, C));
+    // column-unit stream (wide pair tiles; tile knob nstream=1): every pair gets an equal
+    // share of 128-column units, whole K — balance without stream-K's partial-sum fixup
+    P.vmode = 0;
+    if (s->nw == 512 && CL == 2 && p.tiles.nstream == 1) {
+      P.vmode = 1;
+      P.sk_pairs = 0;
+      P.nfull = 0;
+      P.ups = (int)((P.N + 127) / 128);
+      P.vunits = (int64_t)P.tiles_m * P.ups;
+      P.idesc128 = (P.idesc & ~(0x3Fu << 17)) | ((uint32_t)(128 >> 3) << 17);
+    }
+    const int clusters = P.vmode ? (int)std::min<int64_t>(C, P.vunits)
+                                 : (P.sk_pairs > 0 ? C : std::max(1, std::min(T, C)));
     P.trace_n = clusters * NPP * (T / clusters + 4);
     P.trace = t4_trace_buffer(P.trace_n);
     if (!P.trace) P.trace_n = 0;

@@ -620,6 +620,31 @@ def test_t4_stream_k(shape, tile, kind):
         assert np.all(got[0] == float(K))
 
 
+@pytest.mark.parametrize("shape,bt", [((4096, 4096, 4096), False), ((512, 4096, 4096), False), ((700, 1000, 1000), False),
+                                      ((300, 1000, 512), True), ((12544, 512, 1024), False), ((256, 384, 128), True)])
+def test_t4_column_unit_stream(shape, bt):
+    """Wide 2-SM pair tiles under the column-unit stream schedule (tile knob nstream=1):
+    every pair takes an equal share of 128-column units of 256-row strips, whole K, as
+    tiles of 1-4 units (an odd last unit runs as an N = 128 MMA with 64 columns per CTA);
+    ragged M / N, MN-major and K-major B; repeatable bit for bit."""
+    M, N, K = shape
+    spec = _mm_spec(M, N, K, False, bt)
+    x = G.gen_inputs(spec, 3150, "positive")
+    plan = None
+    first = None
+    for _ in range(2):
+        got, plan = run_gpu(spec, x, plan=plan, force_tile="bn=512,nstream=1,split=1")
+        assert plan.describe()["t4_variant"] & 8
+        if M * N <= 1000 * 1000:
+            assert_close_full(spec, x, got, 1e-2, kind="rel")
+        else:
+            assert_close_points(spec, x, got, 1e-2, n=20000, kind="rel")
+        if first is None:
+            first = got[0].copy()
+        else:
+            assert np.array_equal(first, got[0])
+
+
 @pytest.mark.parametrize("shape,out", [((100, 300, 4096), "f32"), ((100, 300, 4096), "bf16"), ((64, 512, 2048), "f32")])
 def test_t4_few_tile_splitk(shape, out):
     """1-SM kernel with few tiles and a deep K (as MCC conv5_1 at N = 1): every tile is split
