@@ -73,6 +73,7 @@ struct Tiles {
   int epi = 0;                        // T4 scatter epilogue: 0 auto, 1 never the bulk-run (EPI 3) kernel
   int krot = 0;                       // T4 k-block rotation per tile (1 = on)
   int l2pf = 0;                       // T1 7-point row loads: L2 prefetch hint 0 none, 1 128 B, 2 256 B
+  int areuse = -1;                    // T4 2-SM wide: k-outer MMA order reusing A from the collector (-1 auto = on, 0 off)
   int nstream = -1;                   // T4 2-SM wide: column-unit stream schedule (-1 auto, 0 off, 1 on)
   std::string source = "default";
 };

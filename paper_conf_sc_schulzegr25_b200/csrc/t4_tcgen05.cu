@@ -105,6 +105,7 @@ struct Params {
   // 128-column units (ups per strip, vunits in all); pair p owns units
   // [p·vunits/npairs, (p+1)·vunits/npairs) — whole K, no partial sums — as tiles of ≤ 4
   // units that never cross a strip, so the pairs' work differs by at most one unit
+  int areuse;                       // wide tiles: k-outer MMA order with A kept in the collector
   int vmode, ups;
   int64_t vunits;
   uint32_t idesc128;                // the N = 128 instruction descriptor (a tile's odd last unit)
@@ -974,6 +975,20 @@ __device__ __forceinline__ void mma_bf16_cg2(uint32_t d_tmem, uint64_t a, uint64
       "tcgen05.mma.cta_group::2.kind::f16 [%0], %1, %2, %3, p;\n\t}" ::"r"(d_tmem),
       "l"(a), "l"(b), "r"(idesc), "r"(acc));
 }
+// the same MMA keeping its A operand in the tensor core's collector buffer (A_KEEP) for the
+// next MMA, which reads it from there (A_REUSE) instead of from shared memory
+__device__ __forceinline__ void mma_bf16_cg2_afill(uint32_t d_tmem, uint64_t a, uint64_t b, uint32_t idesc, uint32_t acc) {
+  asm volatile(
+      "{\n\t.reg .pred p;\n\tsetp.ne.b32 p, %4, 0;\n\t"
+      "tcgen05.mma.cta_group::2.kind::f16.collector::a::fill [%0], %1, %2, %3, p;\n\t}" ::"r"(d_tmem),
+      "l"(a), "l"(b), "r"(idesc), "r"(acc));
+}
+__device__ __forceinline__ void mma_bf16_cg2_alast(uint32_t d_tmem, uint64_t a, uint64_t b, uint32_t idesc, uint32_t acc) {
+  asm volatile(
+      "{\n\t.reg .pred p;\n\tsetp.ne.b32 p, %4, 0;\n\t"
+      "tcgen05.mma.cta_group::2.kind::f16.collector::a::lastuse [%0], %1, %2, %3, p;\n\t}" ::"r"(d_tmem),
+      "l"(a), "l"(b), "r"(idesc), "r"(acc));
+}
 // commit to the barrier at `bar`'s offset in every CTA of `mask` (cluster ranks)
 __device__ __forceinline__ void mma_commit_cg2_mask(uint32_t bar, uint16_t mask) {
   asm volatile("tcgen05.commit.cta_group::2.mbarrier::arrive::one.shared::cluster.multicast::cluster.b64 [%0], %1;" ::"r"(bar),
@@ -1158,8 +1173,9 @@ __global__ void __cluster_dims__(CL, 1, 1) __launch_bounds__(THREADS, 1)
           tc_fence_after();
         }
         const uint32_t d = tmem + acc * BN;
-        long long wfull = 0;
+        long long wfull = 0, cfirst = 0;
         for (int kb = kb0; kb < kb1; ++kb) {
+          if (P.trace && kb == kb0) cfirst = clock64();
           if (P.trace) {
             const long long c0 = clock64();
             mbar_wait(full0 + 8 * stage, phase);
@@ -1174,6 +1190,30 @@ __global__ void __cluster_dims__(CL, 1, 1) __launch_bounds__(THREADS, 1)
           }
           const uint32_t a0 = smem_u32(sA + stage * A2_BYTES), b0 = smem_u32(sB + stage * BSTG);
           const int mnh = P.vmode ? (w.nu + 1) / 2 : NH;
+          if (NH == 2 && P.areuse && !P.vmode) {
+            // k-outer: the two column halves' MMAs of one 16-deep k slice share A, read from
+            // shared memory once (collector fill) and reused by the second MMA
+            if (kb == kb0) {
+#pragma unroll
+              for (int h = 0; h < 2; ++h) {
+                const long long ch = P.trace ? clock64() : 0;
+                mbar_wait(tempty0 + 8 * h, (it & 1) ^ 1);
+                if (P.trace && pair_gid + u * nclusters * NPP < P.trace_n)
+                  P.trace[8 * (pair_gid + u * nclusters * NPP) + 5] += (unsigned long long)(clock64() - ch);
+              }
+              tc_fence_after();
+            }
+#pragma unroll
+            for (int k = 0; k < BK / 16; ++k) {
+              const uint64_t ad = P.a_mn_major ? sdesc(a0 + 2048 * k, 8192, 1024) : sdesc(a0 + 32 * k, 16, 1024);
+              const uint64_t bd0 = P.b_mn_major ? sdesc(b0 + 2048 * k, 8192, 1024) : sdesc(b0 + 32 * k, 16, 1024);
+              const uint64_t bd1 = P.b_mn_major ? sdesc(b0 + B2_BYTES + 2048 * k, 8192, 1024)
+                                                : sdesc(b0 + B2_BYTES + 32 * k, 16, 1024);
+              const uint32_t accf = (kb != kb0) || k != 0;
+              mma_bf16_cg2_afill(d, ad, bd0, P.idesc, accf);
+              mma_bf16_cg2_alast(d + 256, ad, bd1, P.idesc, accf);
+            }
+          } else
 #pragma unroll
           for (int h = 0; h < NH; ++h) {
             if (h >= mnh) break;
@@ -1200,7 +1240,10 @@ __global__ void __cluster_dims__(CL, 1, 1) __launch_bounds__(THREADS, 1)
         mma_commit_cg2_mask(tfull0 + 8 * acc, (uint16_t)(3u << (2 * pp)));
         if (P.trace && pair_gid + u * nclusters * NPP < P.trace_n) {
           P.trace[8 * (pair_gid + u * nclusters * NPP) + 2] = gtimer();
-          P.trace[8 * (pair_gid + u * nclusters * NPP) + 4] = (unsigned long long)wfull;
+          // low word: cycles waiting for full stages; high word: cycles from the first wait to
+          // the last MMA issued (the SM clock of this tile follows from mma_us)
+          P.trace[8 * (pair_gid + u * nclusters * NPP) + 4] =
+              (unsigned long long)(wfull & 0xffffffffll) | ((unsigned long long)(clock64() - cfirst) << 32);
         }
       }
       // drain: the last accumulators must be released before the barriers go away
@@ -2303,6 +2346,7 @@ mdh_status launch_t4(const Plan& p, const void* const* in, void* const* out, voi
     }
     // column-unit stream (wide pair tiles; tile knob nstream=1): every pair gets an equal
     // share of 128-column units, whole K — balance without stream-K's partial-sum fixup
+    P.areuse = s->nw == 512 && p.tiles.areuse != 0;
     P.vmode = 0;
     if (s->nw == 512 && CL == 2 && p.tiles.nstream == 1) {
       P.vmode = 1;

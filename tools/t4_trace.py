@@ -51,7 +51,9 @@ def main():
         for u, (sm, pair, a0, a1, e, wf, wa, ts, tp) in enumerate(tr):
             units.append({"u": u, "pair": pair, "sm": sm, "start_us": round((a0 - t0) / 1e3, 2),
                           "mma_us": round((a1 - a0) / 1e3, 2), "epi_done_us": round((e - t0) / 1e3, 2),
-                          "wait_full_kcyc": round(wf / 1e3, 1), "wait_acc_kcyc": round(wa / 1e3, 1),
+                          "wait_full_kcyc": round((wf & 0xffffffff) / 1e3, 1), "wait_acc_kcyc": round(wa / 1e3, 1),
+                          "issue_kcyc": round((wf >> 32) / 1e3, 1),
+                          "mhz": round((wf >> 32) / ((a1 - a0) / 1e3), 0) if a1 > a0 else None,
                           "seen_us": round((ts - t0) / 1e3, 2) if ts else None,
                           "published_us": round((tp - t0) / 1e3, 2) if tp else None})
         pairs = {}
