@@ -880,8 +880,9 @@ __global__ void __launch_bounds__(AG ? THREADS + AG_THREADS : THREADS, 1)
 // first and finishers last, so a finisher finds its partials (nearly always) published;
 // all pairs are co-resident (persistent grid), so the flag waits cannot deadlock.
 struct SkWork { int t, kb0, kb1, role, u0, nu; };   // u0 / nu: first column unit and units (vmode)
+template <bool LEAN = false>
 struct SkIter {
-  int u, step, nfull, kb, ups;
+  int u, step, nfull, kb, ups, tiles_n;
   bool vmode;
   int64_t k, e;
   __device__ __forceinline__ SkIter(const Params& P, int pair, int npairs) {
@@ -889,13 +890,15 @@ struct SkIter {
     step = npairs;
     nfull = P.nfull;
     kb = P.num_kb;
-    vmode = P.vmode != 0;
+    vmode = !LEAN && P.vmode != 0;
     ups = P.ups;
+    tiles_n = P.tiles_n;
     k = e = 0;
-    if (vmode) {
-      k = (int64_t)pair * P.vunits / npairs;
-      e = (int64_t)(pair + 1) * P.vunits / npairs;
-    } else if (P.sk_pairs > 0 && pair < P.sk_pairs) {
+    if (vmode) {                     // column units after the nfull whole 256×512 tiles
+      const int64_t g0 = nfull > 0 ? (int64_t)(nfull / tiles_n) * ups + 4 * (nfull % tiles_n) : 0;
+      k = g0 + (int64_t)pair * (P.vunits - g0) / npairs;
+      e = g0 + (int64_t)(pair + 1) * (P.vunits - g0) / npairs;
+    } else if (!LEAN && P.sk_pairs > 0 && pair < P.sk_pairs) {
       k = (int64_t)pair * P.sk_w / P.sk_pairs;
       e = (int64_t)(pair + 1) * P.sk_w / P.sk_pairs;
     }
@@ -903,7 +906,13 @@ struct SkIter {
   __device__ __forceinline__ bool next(SkWork* w) {
     w->u0 = 0;
     w->nu = 0;
-    if (vmode) {                     // units k … e-1: strip k / ups, ≤ 4 units per tile
+    if (vmode) {                     // whole tiles, then units k … e-1: strip k / ups, ≤ 4 units per tile
+      if (u < nfull) {
+        const int cu = 4 * (u % tiles_n);
+        w->t = u / tiles_n; w->kb0 = 0; w->kb1 = kb; w->role = 0; w->u0 = cu; w->nu = min(4, ups - cu);
+        u += step;
+        return true;
+      }
       if (k >= e) return false;
       const int strip = (int)(k / ups), cu = (int)(k % ups);
       const int nu = (int)min((int64_t)4, min(e - k, (int64_t)(ups - cu)));
@@ -916,7 +925,7 @@ struct SkIter {
       u += step;
       return true;
     }
-    if (k >= e) return false;
+    if (LEAN || k >= e) return false;
     const int64_t x = k / kb;
     w->t = nfull + (int)x;
     w->kb0 = (int)(k - x * kb);
@@ -1035,11 +1044,15 @@ __device__ __forceinline__ void mbar_arrive_cluster(uint32_t bar_cluster) {
 // single-buffered staging (4 × 48 KB + 32 KB fits the 227 KB budget; tile knob stages=4:
 // MCC conv5_1 +1-3 %, MatMul 4096³ / 8192³ -2 / -3 %: the single staging buffer slows the
 // whole-tile epilogues)
-template <bool OUT_ROWMAJOR, int CL, int NW = 256, int WST = S2W>
+template <bool OUT_ROWMAJOR, int CL, int NW = 256, int WST = S2W, bool LEAN = false>
 __global__ void __cluster_dims__(CL, 1, 1) __launch_bounds__(THREADS, 1)
     gemm2_kernel(const __grid_constant__ CUtensorMap mapA, const __grid_constant__ CUtensorMap mapB,
                  const __grid_constant__ CUtensorMap mapC, const __grid_constant__ Params P) {
   extern __shared__ __align__(1024) uint8_t smem_raw[];
+  // LEAN: whole tiles only (no stream-K roles, no column units, no trace) — a smaller
+  // instance whose hot loops share the instruction cache with less cold code
+  unsigned long long* const trace = LEAN ? nullptr : P.trace;
+  const bool vm = !LEAN && P.vmode != 0;
   constexpr int NH = NW / 256;                   // N=256 MMAs per k-step
   constexpr int NS = NW == 512 ? WST : S2;       // ring stages
   constexpr int EPB = (NW == 512 && WST == 4) ? 1 : 2;   // epilogue staging buffers per warp
@@ -1061,7 +1074,7 @@ __global__ void __cluster_dims__(CL, 1, 1) __launch_bounds__(THREADS, 1)
   // pair tiles: tiles_m/tiles_n count 256×NW tiles; clusters stride over them
   const int cluster_id = blockIdx.x / CL, nclusters = gridDim.x / CL;
   const int pair_gid = cluster_id * NPP + (int)pp;   // partial slot / trace row of this pair
-  if (P.trace && threadIdx.x == 0 && pair_gid < 256) P.trace[8 * P.trace_n + 2 * pair_gid + rank * 512] = gtimer();
+  if (trace && threadIdx.x == 0 && pair_gid < 256) trace[8 * P.trace_n + 2 * pair_gid + rank * 512] = gtimer();
 
   if (warp == 0 && lane == 0) {
     asm volatile("prefetch.tensormap [%0];" ::"l"((uint64_t)&mapA) : "memory");
@@ -1093,17 +1106,17 @@ __global__ void __cluster_dims__(CL, 1, 1) __launch_bounds__(THREADS, 1)
       // ===== TMA producer (both CTAs; bytes are counted at the leader's full barrier) =====
       int stage = 0;
       uint32_t phase = 0;
-      SkIter wi(P, cluster_id, nclusters);
+      SkIter<LEAN> wi(P, cluster_id, nclusters);
       SkWork w;
       while (wi.next(&w)) {
         const int t = w.t, kb0 = w.kb0, kb1 = w.kb1;
-        const int m0 = P.vmode ? t * 256 + (int)rank * 128 : ((t / P.tiles_n) * NPP + (int)pp) * 256 + (int)rank * 128;
-        const int n0 = P.vmode ? 128 * w.u0 + (int)rank * 128 : (t % P.tiles_n) * NW + (int)rank * 128;
+        const int m0 = vm ? t * 256 + (int)rank * 128 : ((t / P.tiles_n) * NPP + (int)pp) * 256 + (int)rank * 128;
+        const int n0 = vm ? 128 * w.u0 + (int)rank * 128 : (t % P.tiles_n) * NW + (int)rank * 128;
         // vmode: MMA h covers units u0+2h, u0+2h+1 (N = 256, 128 columns per CTA) or only the
         // tile's odd last unit (N = 128, 64 columns per CTA: one 64-column MN-major box)
         const int vnh = (w.nu + 1) / 2;
         const bool vodd = (w.nu & 1) != 0;
-        const uint32_t bbytes = !P.vmode ? (uint32_t)BSTG
+        const uint32_t bbytes = !vm ? (uint32_t)BSTG
                                          : (uint32_t)(vnh * B2_BYTES - (vodd && P.b_mn_major ? B2_BYTES / 2 : 0));
         for (int kb = kb0; kb < kb1; ++kb) {
           mbar_wait(empty0 + 8 * stage, phase ^ 1);
@@ -1127,7 +1140,7 @@ __global__ void __cluster_dims__(CL, 1, 1) __launch_bounds__(THREADS, 1)
             const uint16_t mask = (uint16_t)((1u << rank) | (1u << (2 + rank)));
             if (P.b_mn_major) tma_load_2d_cg2_mc(b_dst + pp * 8192, &mapB, fb_leader, n0 + 64 * pp, k0, mask);
             else tma_load_2d_cg2_mc(b_dst + pp * 8192, &mapB, fb_leader, k0, n0 + 64 * pp, mask);
-          } else if (P.vmode) {
+          } else if (vm) {
             for (int h = 0; h < vnh; ++h) {
               const bool half_unit = vodd && h == vnh - 1;     // N = 128: 64 columns per CTA
               const int nb = half_unit ? 128 * (w.u0 + 2 * h) + (int)rank * 64 : n0 + 256 * h;
@@ -1159,24 +1172,24 @@ __global__ void __cluster_dims__(CL, 1, 1) __launch_bounds__(THREADS, 1)
       int stage = 0;
       uint32_t phase = 0;
       int it = 0;
-      SkIter wi(P, cluster_id, nclusters);
+      SkIter<LEAN> wi(P, cluster_id, nclusters);
       SkWork w;
       for (; wi.next(&w); ++it) {
         const int u = it;
         const int kb0 = w.kb0, kb1 = w.kb1;
         const int acc = NH == 1 ? it & 1 : 0;
-        const long long ct0 = P.trace ? clock64() : 0;
+        const long long ct0 = trace ? clock64() : 0;
         if (NH == 1) {
           mbar_wait(tempty0 + 8 * acc, ((it >> 1) & 1) ^ 1);
-          if (P.trace && pair_gid + u * nclusters * NPP < P.trace_n)
-            P.trace[8 * (pair_gid + u * nclusters * NPP) + 5] = (unsigned long long)(clock64() - ct0);
+          if (trace && pair_gid + u * nclusters * NPP < P.trace_n)
+            trace[8 * (pair_gid + u * nclusters * NPP) + 5] = (unsigned long long)(clock64() - ct0);
           tc_fence_after();
         }
         const uint32_t d = tmem + acc * BN;
         long long wfull = 0, cfirst = 0;
         for (int kb = kb0; kb < kb1; ++kb) {
-          if (P.trace && kb == kb0) cfirst = clock64();
-          if (P.trace) {
+          if (trace && kb == kb0) cfirst = clock64();
+          if (trace) {
             const long long c0 = clock64();
             mbar_wait(full0 + 8 * stage, phase);
             wfull += clock64() - c0;
@@ -1184,22 +1197,22 @@ __global__ void __cluster_dims__(CL, 1, 1) __launch_bounds__(THREADS, 1)
             mbar_wait(full0 + 8 * stage, phase);
           }
           tc_fence_after();
-          if (P.trace && kb == kb0 && pair_gid + u * nclusters * NPP < P.trace_n) {
-            P.trace[8 * (pair_gid + u * nclusters * NPP)] = ((unsigned long long)smid() << 32) | (unsigned)pair_gid;
-            P.trace[8 * (pair_gid + u * nclusters * NPP) + 1] = gtimer();
+          if (trace && kb == kb0 && pair_gid + u * nclusters * NPP < P.trace_n) {
+            trace[8 * (pair_gid + u * nclusters * NPP)] = ((unsigned long long)smid() << 32) | (unsigned)pair_gid;
+            trace[8 * (pair_gid + u * nclusters * NPP) + 1] = gtimer();
           }
           const uint32_t a0 = smem_u32(sA + stage * A2_BYTES), b0 = smem_u32(sB + stage * BSTG);
-          const int mnh = P.vmode ? (w.nu + 1) / 2 : NH;
-          if (NH == 2 && P.areuse && !P.vmode) {
+          const int mnh = vm ? (w.nu + 1) / 2 : NH;
+          if (NH == 2 && P.areuse && mnh == 2) {
             // k-outer: the two column halves' MMAs of one 16-deep k slice share A, read from
             // shared memory once (collector fill) and reused by the second MMA
             if (kb == kb0) {
 #pragma unroll
               for (int h = 0; h < 2; ++h) {
-                const long long ch = P.trace ? clock64() : 0;
+                const long long ch = trace ? clock64() : 0;
                 mbar_wait(tempty0 + 8 * h, (it & 1) ^ 1);
-                if (P.trace && pair_gid + u * nclusters * NPP < P.trace_n)
-                  P.trace[8 * (pair_gid + u * nclusters * NPP) + 5] += (unsigned long long)(clock64() - ch);
+                if (trace && pair_gid + u * nclusters * NPP < P.trace_n)
+                  trace[8 * (pair_gid + u * nclusters * NPP) + 5] += (unsigned long long)(clock64() - ch);
               }
               tc_fence_after();
             }
@@ -1211,18 +1224,18 @@ __global__ void __cluster_dims__(CL, 1, 1) __launch_bounds__(THREADS, 1)
                                                 : sdesc(b0 + B2_BYTES + 32 * k, 16, 1024);
               const uint32_t accf = (kb != kb0) || k != 0;
               mma_bf16_cg2_afill(d, ad, bd0, P.idesc, accf);
-              mma_bf16_cg2_alast(d + 256, ad, bd1, P.idesc, accf);
+              mma_bf16_cg2_alast(d + 256, ad, bd1, (vm && (w.nu & 1)) ? P.idesc128 : P.idesc, accf);
             }
           } else
 #pragma unroll
           for (int h = 0; h < NH; ++h) {
             if (h >= mnh) break;
-            const uint32_t idesc_h = (P.vmode && (w.nu & 1) && h == mnh - 1) ? P.idesc128 : P.idesc;
+            const uint32_t idesc_h = (vm && (w.nu & 1) && h == mnh - 1) ? P.idesc128 : P.idesc;
             if (NH > 1 && kb == kb0) {      // column half h of the accumulator drained?
-              const long long ch = P.trace ? clock64() : 0;
+              const long long ch = trace ? clock64() : 0;
               mbar_wait(tempty0 + 8 * h, (it & 1) ^ 1);
-              if (P.trace && pair_gid + u * nclusters * NPP < P.trace_n)
-                P.trace[8 * (pair_gid + u * nclusters * NPP) + 5] += (unsigned long long)(clock64() - ch);
+              if (trace && pair_gid + u * nclusters * NPP < P.trace_n)
+                trace[8 * (pair_gid + u * nclusters * NPP) + 5] += (unsigned long long)(clock64() - ch);
               tc_fence_after();
             }
 #pragma unroll
@@ -1238,11 +1251,11 @@ __global__ void __cluster_dims__(CL, 1, 1) __launch_bounds__(THREADS, 1)
           if (++stage == NS) { stage = 0; phase ^= 1; }
         }
         mma_commit_cg2_mask(tfull0 + 8 * acc, (uint16_t)(3u << (2 * pp)));
-        if (P.trace && pair_gid + u * nclusters * NPP < P.trace_n) {
-          P.trace[8 * (pair_gid + u * nclusters * NPP) + 2] = gtimer();
+        if (trace && pair_gid + u * nclusters * NPP < P.trace_n) {
+          trace[8 * (pair_gid + u * nclusters * NPP) + 2] = gtimer();
           // low word: cycles waiting for full stages; high word: cycles from the first wait to
           // the last MMA issued (the SM clock of this tile follows from mma_us)
-          P.trace[8 * (pair_gid + u * nclusters * NPP) + 4] =
+          trace[8 * (pair_gid + u * nclusters * NPP) + 4] =
               (unsigned long long)(wfull & 0xffffffffll) | ((unsigned long long)(clock64() - cfirst) << 32);
         }
       }
@@ -1268,16 +1281,17 @@ __global__ void __cluster_dims__(CL, 1, 1) __launch_bounds__(THREADS, 1)
     int sbuf = 0;                                  // staging buffer of the next TMA store
     const uint32_t tempty_leader = map_to_rank(tempty0, 2 * pp);
     int it = 0;
-    SkIter wi(P, cluster_id, nclusters);
+    SkIter<LEAN> wi(P, cluster_id, nclusters);
     SkWork w;
     for (; wi.next(&w); ++it) {
       const int t = w.t;
+      const int role = LEAN ? 0 : w.role;
       const int acc = NH == 1 ? it & 1 : 0;
-      const int64_t m = P.vmode ? (int64_t)t * 256 + rank * 128 + row
+      const int64_t m = vm ? (int64_t)t * 256 + rank * 128 + row
                                 : ((int64_t)(t / P.tiles_n) * NPP + pp) * 256 + rank * 128 + row;
-      const int64_t ntile = P.vmode ? (int64_t)128 * w.u0 : (int64_t)(t % P.tiles_n) * NW;
+      const int64_t ntile = vm ? (int64_t)128 * w.u0 : (int64_t)(t % P.tiles_n) * NW;
       // columns of this tile held by this warp group in MMA half h (vmode: a group may hold none)
-      auto group_has = [&](int h) { return !P.vmode || 2 * h + half < w.nu; };
+      auto group_has = [&](int h) { return !vm || 2 * h + half < w.nu; };
       mbar_wait(tfull0 + 8 * acc, NH == 1 ? (it >> 1) & 1 : it & 1);
       tc_fence_after();
       const bool mok = m < P.M;
@@ -1286,7 +1300,7 @@ __global__ void __cluster_dims__(CL, 1, 1) __launch_bounds__(THREADS, 1)
       // float4 [c][j][lane] (each store / load instruction covers 512 contiguous bytes)
       float4* mine = reinterpret_cast<float4*>(P.skpart + (int64_t)pair_gid * (NH * 65536) + ew * (NH * 4096)) + lane;
       int q1 = cluster_id;                           // finisher: partials of pairs cluster_id+1 .. q1
-      if (w.role == 2) {
+      if (role == 2) {
         const int64_t tend = (int64_t)(t - P.nfull + 1) * P.num_kb;
         while (q1 + 1 < P.sk_pairs && (int64_t)(q1 + 1) * P.sk_w / P.sk_pairs < tend) ++q1;
         if (lane == 0)
@@ -1294,8 +1308,8 @@ __global__ void __cluster_dims__(CL, 1, 1) __launch_bounds__(THREADS, 1)
             while (*((volatile unsigned*)(P.skflag + (q * NPP + pp) * 16 + ew)) == 0u) __nanosleep(64);
         __syncwarp();
         __threadfence();
-        if (P.trace && leader && warp == 2 && lane == 0 && pair_gid + it * nclusters * NPP < P.trace_n)
-          P.trace[8 * (pair_gid + it * nclusters * NPP) + 6] = gtimer();
+        if (trace && leader && warp == 2 && lane == 0 && pair_gid + it * nclusters * NPP < P.trace_n)
+          trace[8 * (pair_gid + it * nclusters * NPP) + 6] = gtimer();
       }
       auto epi_chunk = [&](uint32_t* r, int64_t nb, int pc) {
         // fold the producers' partials in k order, two partials' loads in flight at a time
@@ -1332,7 +1346,7 @@ __global__ void __cluster_dims__(CL, 1, 1) __launch_bounds__(THREADS, 1)
             r[4 * j + 3] = __float_as_uint(__uint_as_float(r[4 * j + 3]) + b.w);
           }
         }
-        if (OUT_ROWMAJOR && P.c_vec4) {
+        if (LEAN || (OUT_ROWMAJOR && P.c_vec4)) {   // (LEAN launches only with the TMA store map)
           // this warp's 32 rows × 32 columns into a 128B-swizzled staging image (16-byte chunk
           // j of row r at (j ^ (r & 7))·16: conflict-free), then one TMA tensor store of the
           // 32×32 box (rows / columns beyond M / N are clipped by the TMA unit); two staging
@@ -1388,7 +1402,7 @@ __global__ void __cluster_dims__(CL, 1, 1) __launch_bounds__(THREADS, 1)
         tmem_ld32(tb + c * 32, r);
         const int64_t nb = n0 + c * 32;
         const int pc = h * 4 + c;                    // 32-column chunk index in the partial
-        if (w.role == 1) {
+        if (role == 1) {
 #pragma unroll
           for (int j = 0; j < 8; ++j)
             mine[(pc * 8 + j) * 32] = make_float4(__uint_as_float(r[4 * j]), __uint_as_float(r[4 * j + 1]),
@@ -1403,13 +1417,13 @@ __global__ void __cluster_dims__(CL, 1, 1) __launch_bounds__(THREADS, 1)
         if (lane == 0) mbar_arrive_cluster(tempty_leader + 8 * h);
       }
       }
-      if (w.role == 1) {               // publish this warp's part of the partial tile
+      if (role == 1) {               // publish this warp's part of the partial tile
         __threadfence();
         __syncwarp();
         if (lane == 0) atomicExch(P.skflag + pair_gid * 16 + ew, 1u);
-        if (P.trace && leader && warp == 2 && lane == 0 && pair_gid + it * nclusters * NPP < P.trace_n)
-          P.trace[8 * (pair_gid + it * nclusters * NPP) + 7] = gtimer();
-      } else if (w.role == 2 && lane == 0) {
+        if (trace && leader && warp == 2 && lane == 0 && pair_gid + it * nclusters * NPP < P.trace_n)
+          trace[8 * (pair_gid + it * nclusters * NPP) + 7] = gtimer();
+      } else if (role == 2 && lane == 0) {
         for (int q = cluster_id + 1; q <= q1; ++q) P.skflag[(q * NPP + pp) * 16 + ew] = 0u;   // consumed: back to rest
       }
       if (NH == 1) {
@@ -1417,8 +1431,8 @@ __global__ void __cluster_dims__(CL, 1, 1) __launch_bounds__(THREADS, 1)
         __syncwarp();
         if (lane == 0) mbar_arrive_cluster(tempty_leader + 8 * acc);
       }
-      if (P.trace && leader && warp == 2 && lane == 0 && pair_gid + it * nclusters * NPP < P.trace_n)
-        P.trace[8 * (pair_gid + it * nclusters * NPP) + 3] = gtimer();
+      if (trace && leader && warp == 2 && lane == 0 && pair_gid + it * nclusters * NPP < P.trace_n)
+        trace[8 * (pair_gid + it * nclusters * NPP) + 3] = gtimer();
     }
     if (lane == 0) asm volatile("cp.async.bulk.wait_group 0;" ::: "memory");   // stores done before exit
   }
@@ -1429,7 +1443,7 @@ __global__ void __cluster_dims__(CL, 1, 1) __launch_bounds__(THREADS, 1)
     tc_fence_after();
     asm volatile("tcgen05.dealloc.cta_group::2.sync.aligned.b32 %0, %1;" ::"r"(tmem), "r"(TMEM_COLS));
   }
-  if (P.trace && threadIdx.x == 0 && pair_gid < 256) P.trace[8 * P.trace_n + 2 * pair_gid + 1 + rank * 512] = gtimer();
+  if (trace && threadIdx.x == 0 && pair_gid < 256) trace[8 * P.trace_n + 2 * pair_gid + 1 + rank * 512] = gtimer();
 }
 
 // Few-tile split-K (1-SM kernel, P.xfold): S splits of each of the T tiles wrote dense
@@ -1653,7 +1667,7 @@ struct T4State {
   int cg = 1;      // 1: one SM per 128×256 tile; 2: SM pair per 256×256 tile
   int cl = 2;      // 2-SM kernel: CTAs per cluster (4: two pairs share B by multicast)
   int nw = 256;    // 2-SM kernel: N extent of a pair tile (512: two MMAs per k-step)
-  int wst = 3;     // wide 2-SM ring stages (4: single-buffered epilogue staging; tile knob stages=4)
+  int wst = 4;     // wide 2-SM ring stages (4: single-buffered epilogue staging; tile knob stages=3: double-buffered)
   bool sk_ok = false;   // 2-SM kernel: stream-K workspace reserved
   bool ag = false; // A staged by the kernel's gather warps (no A tensor map, no pre-pass)
   bool ic = false;  // A through a TMA im2col map
@@ -1798,7 +1812,7 @@ mdh_status prepare_t4(Plan* p) {
   if (prepare_t4_conv(p)) return MDH_OK;           // small-K direct variant (t4_conv.cu)
   const Contraction& c = p->con;
   T4State* s = new T4State();
-  s->wst = p->tiles.stages == 4 ? 4 : 3;
+  s->wst = p->tiles.stages == 3 ? 3 : 4;
   size_t ws = 0;
   std::string w2;
   const t4::Layout2D a_direct = t4::operand_layout(*p, c.md, c.nm, c.M, p->in[c.a_buf].acc[0], &w2, "A");
@@ -2274,9 +2288,11 @@ mdh_status launch_t4(const Plan& p, const void* const* in, void* const* out, voi
                                            (int)(t4::SMEM_LIMIT - t4::BN * sizeof(int64_t)));
       if (e != cudaSuccess) attr_err = e;
     }
-    const void* k2[6] = {(const void*)t4::gemm2_kernel<true, 2>, (const void*)t4::gemm2_kernel<false, 2>,
-                         (const void*)t4::gemm2_kernel<true, 4>, (const void*)t4::gemm2_kernel<false, 4>,
-                         (const void*)t4::gemm2_kernel<true, 2, 512>, (const void*)t4::gemm2_kernel<true, 2, 512, 4>};
+    const void* k2[] = {(const void*)t4::gemm2_kernel<true, 2>, (const void*)t4::gemm2_kernel<true, 4>,
+                        (const void*)t4::gemm2_kernel<true, 2, 512>, (const void*)t4::gemm2_kernel<true, 2, 512, 4>,
+                        (const void*)t4::gemm2_kernel<true, 2, 256, t4::S2W, true>,
+                        (const void*)t4::gemm2_kernel<true, 2, 512, 3, true>,
+                        (const void*)t4::gemm2_kernel<true, 2, 512, 4, true>};
     for (const void* k : k2) {
       cudaError_t e = cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, t4::SMEM2_BYTES);
       if (e != cudaSuccess) attr_err = e;
@@ -2348,10 +2364,12 @@ mdh_status launch_t4(const Plan& p, const void* const* in, void* const* out, voi
     // share of 128-column units, whole K — balance without stream-K's partial-sum fixup
     P.areuse = s->nw == 512 && p.tiles.areuse != 0;
     P.vmode = 0;
-    if (s->nw == 512 && CL == 2 && p.tiles.nstream == 1) {
+    if (s->nw == 512 && CL == 2 && (p.tiles.nstream == 1 || (p.tiles.nstream == 2 && T > C && T % C != 0))) {
+      // nstream=2: the complete waves run whole tiles, only the partial last wave is cut
+      // into column units (no partial sums: every piece runs the whole K)
       P.vmode = 1;
       P.sk_pairs = 0;
-      P.nfull = 0;
+      P.nfull = p.tiles.nstream == 2 ? (T / C) * C : 0;
       P.ups = (int)((P.N + 127) / 128);
       P.vunits = (int64_t)P.tiles_m * P.ups;
       P.idesc128 = (P.idesc & ~(0x3Fu << 17)) | ((uint32_t)(128 >> 3) << 17);
@@ -2378,7 +2396,15 @@ mdh_status launch_t4(const Plan& p, const void* const* in, void* const* out, voi
                       CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
       if (r != CUDA_SUCCESS) { set_error("cuTensorMapEncodeTiled (C store map) failed (%d)", (int)r); return MDH_ERR_CUDA; }
     }
-    if (s->nw == 512 && s->wst == 4)
+    // whole tiles only: the lean instance (no stream-K / column-unit / trace code)
+    const bool lean = P.sk_pairs == 0 && !P.vmode && !P.trace && CL == 2 && P.c_vec4;
+    if (lean && s->nw == 512 && s->wst == 4)
+      t4::gemm2_kernel<true, 2, 512, 4, true><<<grid2, t4::THREADS, t4::SMEM2_BYTES, st>>>(ma, mb, mc, P);
+    else if (lean && s->nw == 512)
+      t4::gemm2_kernel<true, 2, 512, 3, true><<<grid2, t4::THREADS, t4::SMEM2_BYTES, st>>>(ma, mb, mc, P);
+    else if (lean)
+      t4::gemm2_kernel<true, 2, 256, t4::S2W, true><<<grid2, t4::THREADS, t4::SMEM2_BYTES, st>>>(ma, mb, mc, P);
+    else if (s->nw == 512 && s->wst == 4)
       t4::gemm2_kernel<true, 2, 512, 4><<<grid2, t4::THREADS, t4::SMEM2_BYTES, st>>>(ma, mb, mc, P);
     else if (s->nw == 512) t4::gemm2_kernel<true, 2, 512><<<grid2, t4::THREADS, t4::SMEM2_BYTES, st>>>(ma, mb, mc, P);
     else if (CL == 4) t4::gemm2_kernel<true, 4><<<grid2, t4::THREADS, t4::SMEM2_BYTES, st>>>(ma, mb, mc, P);

@@ -620,12 +620,16 @@ def test_t4_stream_k(shape, tile, kind):
         assert np.all(got[0] == float(K))
 
 
-@pytest.mark.parametrize("shape,bt", [((4096, 4096, 4096), False), ((512, 4096, 4096), False), ((700, 1000, 1000), False),
-                                      ((300, 1000, 512), True), ((12544, 512, 1024), False), ((256, 384, 128), True)])
-def test_t4_column_unit_stream(shape, bt):
+@pytest.mark.parametrize("shape,bt,ns", [((4096, 4096, 4096), False, 1), ((512, 4096, 4096), False, 1),
+                                         ((700, 1000, 1000), False, 1), ((300, 1000, 512), True, 1),
+                                         ((12544, 512, 1024), False, 1), ((256, 384, 128), True, 1),
+                                         ((4096, 4096, 4096), False, 2), ((2500, 4000, 256), False, 2),
+                                         ((2560, 4096, 320), True, 2), ((2500, 3900, 200), True, 2)])
+def test_t4_column_unit_stream(shape, bt, ns):
     """Wide 2-SM pair tiles under the column-unit stream schedule (tile knob nstream=1):
     every pair takes an equal share of 128-column units of 256-row strips, whole K, as
     tiles of 1-4 units (an odd last unit runs as an N = 128 MMA with 64 columns per CTA);
+    nstream=2: whole tiles for the complete waves, units only in the partial last wave;
     ragged M / N, MN-major and K-major B; repeatable bit for bit."""
     M, N, K = shape
     spec = _mm_spec(M, N, K, False, bt)
@@ -633,7 +637,7 @@ def test_t4_column_unit_stream(shape, bt):
     plan = None
     first = None
     for _ in range(2):
-        got, plan = run_gpu(spec, x, plan=plan, force_tile="bn=512,nstream=1,split=1")
+        got, plan = run_gpu(spec, x, plan=plan, force_tile=f"bn=512,nstream={ns},split=1")
         assert plan.describe()["t4_variant"] & 8
         if M * N <= 1000 * 1000:
             assert_close_full(spec, x, got, 1e-2, kind="rel")

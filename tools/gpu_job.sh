@@ -11,7 +11,7 @@
 #   bench[:<bench args>]              python bench.py (default args)                    -> bench.json
 #   ref                               python bench.py --impl reference                  -> ref.json
 #   smoke                             __graft_entry__.smoke()                           -> smoke.log
-#   sweep:<args>                      tools/sweep_tiles.py                              -> sweep.log
+#   sweep:<args>                      tools/sweep_tiles.py (table copy updated)         -> sweep.log, b200.json
 #   py:<script args>                  python <script args>                              -> py.log
 #   torchrun:<N>:<bench args>         torchrun --nproc-per-node N bench.py ...          -> torchrun.log
 set -u
@@ -54,7 +54,8 @@ for step in "$@"; do
       timeout 300 python -c "import __graft_entry__ as g; g.smoke(); print('smoke ok')" > "$OUT/smoke.log" 2>&1
       tail -2 "$OUT/smoke.log" ;;
     sweep)
-      timeout 2400 python tools/sweep_tiles.py $arg > "$OUT/sweep.log" 2>&1; echo "sweep rc=$?"; tail -5 "$OUT/sweep.log" ;;
+      cp tiles/b200.json "$OUT/b200.json"     # the updated table comes back in gpurun_out/
+      timeout 2400 python tools/sweep_tiles.py --out "$OUT/b200.json" $arg > "$OUT/sweep.log" 2>&1; echo "sweep rc=$?"; tail -5 "$OUT/sweep.log" ;;
     py)
       timeout 1200 python $arg >> "$OUT/py.log" 2>&1; echo "py rc=$?"; tail -15 "$OUT/py.log" ;;
     torchrun)

@@ -15,6 +15,9 @@ import sys
 ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
 sys.path.insert(0, ROOT)
 
+T4_WIDE = ["bn=256", "bn=512", "bn=256,split=1", "bn=512,split=1", "bn=512,stages=3", "bn=512,split=1,stages=3"]
+
+
 # (workload, spec builder kwargs, candidates)
 def cases():
     from mdh_workloads import specs as S
@@ -33,19 +36,20 @@ def cases():
         ("prl_B", lambda: (S.prl(1 << 14, 1 << 20), G.prl_inputs(1 << 14, 1 << 20)),
          [f"split={s}" for s in (8, 16, 32, 37, 48, 64)]),
         # T4 2-SM: pair-tile width (256 / 512) × whole tiles vs stream-K for the last wave
+        # (wide tiles: ring stages 4 with one epilogue staging buffer, or 3 with two)
         ("t4_mm_bf16_4096", lambda: (S.matmul(4096, 4096, 4096, "bf16"), G.matmul_inputs(4096, 4096, 4096, "bf16", "signed")),
-         ["bn=256", "bn=512", "bn=256,split=1", "bn=512,split=1"]),
+         T4_WIDE),
         ("t4_mm_bf16_8192", lambda: (S.matmul(8192, 8192, 8192, "bf16"), G.matmul_inputs(8192, 8192, 8192, "bf16", "signed")),
-         ["bn=256", "bn=512", "bn=256,split=1", "bn=512,split=1"]),
+         T4_WIDE),
         ("t4_mm_bf16_2048", lambda: (S.matmul(2048, 2048, 2048, "bf16"), G.matmul_inputs(2048, 2048, 2048, "bf16", "signed")),
-         ["bn=256", "bn=512", "bn=256,split=1", "bn=512,split=1"]),
+         T4_WIDE),
         ("t4_mcc_bf16_conv5_1", lambda: (S.mcc(256, 7, 7, 512, 3, 3, 512, "bf16"),
                                          G.mcc_inputs(S.mcc(256, 7, 7, 512, 3, 3, 512, "bf16"))),
-         ["bn=256", "bn=512", "bn=256,split=1", "bn=512,split=1"]),
+         T4_WIDE),
         # per-rank shapes of the strong-scaled configs (bench.py --gpus N):
         # MatMul 4096³ on M at 2/4/8 GPUs, Jacobi3D 512³ z-slabs, PRL A/B DB slices
         *[(f"rank_mm_bf16_{m}", (lambda m=m: (S.matmul(m, 4096, 4096, "bf16"), G.matmul_inputs(m, 4096, 4096, "bf16", "signed"))),
-           ["bn=256", "bn=512", "bn=256,split=2", "bn=512,split=2", "bn=256,split=1", "bn=512,split=1"])
+           T4_WIDE + ["bn=256,split=2", "bn=512,split=2", "bn=512,split=2,stages=3"])
           for m in (2048, 1024, 512)],
         *[(f"rank_jacobi3d_{z}", (lambda z=z: (S.jacobi3d(z, 512, 512), G.jacobi3d_inputs(z, 512, 512))),
            [f"zchunk={c}" for c in (4, 8, 16, 32)]) for z in (257, 130, 66)],
@@ -74,7 +78,7 @@ def main():
     entries = {(e["template"], e["dtype"], e.get("f"), e.get("op"), tuple(e["bucket"])): e for e in table.get("entries", [])}
     log = []
     for name, mk, cands in cases():
-        if a.only and a.only not in name:
+        if a.only and not any(o in name for o in a.only.split(",")):
             continue
         spec, host = mk()
         tin = None
@@ -111,7 +115,7 @@ def main():
         else:
             # the default won: record the knobs it resolved to (a table entry of {} would
             # fall back to the template defaults, not to the nearest bucket it was timed with)
-            knobs = {"T1_stencil": ("zchunk", "l2pf"), "T2_reduce": ("split",), "T4_tcgen05_contraction": ("bn", "split"),
+            knobs = {"T1_stencil": ("zchunk", "l2pf"), "T2_reduce": ("split",), "T4_tcgen05_contraction": ("bn", "split", "stages"),
                      "T5_prl_pairwise": ("split",), "T3_simt_contraction": ("split",)}.get(d["template"], ())
             tiles = {k: int(d["tiles"][k]) for k in knobs if k in d["tiles"]}
         fname = spec["f"]
