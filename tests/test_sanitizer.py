@@ -17,10 +17,16 @@ def test_compute_sanitizer(tool):
     cs = shutil.which("compute-sanitizer") or "/usr/local/cuda/bin/compute-sanitizer"
     if not os.path.exists(cs):
         pytest.skip("compute-sanitizer not installed")
+    if os.environ.get("MDH_SANITIZER") != "1":
+        # the GPU pool refuses compute-sanitizer (runs under it have left GPUs needing a
+        # reset); opt in with MDH_SANITIZER=1 on a box that allows it
+        pytest.skip("compute-sanitizer runs are opt-in (MDH_SANITIZER=1)")
     cmd = [cs, "--tool", tool, "--error-exitcode", "9", "--target-processes", "all",
            sys.executable, os.path.join(ROOT, "tools", "sanitize_cases.py")]
     r = subprocess.run(cmd, capture_output=True, text=True, timeout=1500, cwd=ROOT)
     out = r.stdout + r.stderr
+    if "closed on this pool" in out:
+        pytest.skip("compute-sanitizer is closed on this GPU pool")
     if tool == "racecheck":
         # The only accepted report: the 2-SM kernel's `tcgen05.alloc.cta_group::2`, where both
         # CTAs of the pair allocate and the hardware writes the (identical) TMEM address into
