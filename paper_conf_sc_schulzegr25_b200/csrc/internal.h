@@ -75,6 +75,8 @@ struct Tiles {
   int l2pf = 0;                       // T1 7-point row loads: L2 prefetch hint 0 none, 1 128 B, 2 256 B
   int areuse = -1;                    // T4 2-SM wide: k-outer MMA order reusing A from the collector (-1 auto = on, 0 off)
   int nstream = -1;                   // T4 2-SM wide: column-unit stream schedule (-1 auto, 0 off, 1 on)
+  int mode = -1;                      // T1 7-point: -1 auto, 0 per-thread rows, 1 warp-coalesced rows,
+                                      // 2 warp-coalesced + y-neighbour rows shared through smem
   std::string source = "default";
 };
 

@@ -523,9 +523,11 @@ std::string describe_plan(const Plan& p) {
     add(", \"contraction\": {\"Z\": %lld, \"M\": %lld, \"N\": %lld, \"K\": %lld, \"nm\": %d, \"nn\": %d, \"nk\": %d, \"nz\": %d}",
         (long long)p.con.Z, (long long)p.con.M, (long long)p.con.N, (long long)p.con.K, p.con.nm, p.con.nn, p.con.nk, p.con.nz);
   add(", \"tiles\": {\"threads\": %d, \"bm\": %d, \"bn\": %d, \"bk\": %d, \"split\": %d, \"stages\": %d, \"vec\": %d, "
-      "\"zchunk\": %d, \"per_thread\": %d, \"cluster\": %d, \"implicit\": %d, \"seg\": %d, \"epi\": %d, \"source\": \"%s\"}",
+      "\"zchunk\": %d, \"per_thread\": %d, \"cluster\": %d, \"implicit\": %d, \"seg\": %d, \"epi\": %d, \"mode\": %d, "
+      "\"source\": \"%s\"}",
       p.tiles.threads, p.tiles.bm, p.tiles.bn, p.tiles.bk, p.tiles.split, p.tiles.stages, p.tiles.vec,
-      p.tiles.zchunk, p.tiles.per_thread, p.tiles.cluster, p.tiles.implicit, p.tiles.seg, p.tiles.epi, p.tiles.source.c_str());
+      p.tiles.zchunk, p.tiles.per_thread, p.tiles.cluster, p.tiles.implicit, p.tiles.seg, p.tiles.epi, p.tiles.mode,
+      p.tiles.source.c_str());
   add(", \"t4_variant\": %d", p.t4_variant);
   add(", \"workspace\": %zu, \"world\": %d, \"rank\": %d, \"shard_dim\": %d, \"shard_is_red\": %s, "
       "\"shard_start\": %lld, \"shard_len\": %lld}",

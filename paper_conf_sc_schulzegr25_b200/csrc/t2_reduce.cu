@@ -252,6 +252,88 @@ __global__ void __launch_bounds__(256) t2_warp_kernel(const __grid_constant__ T2
   }
 }
 
+// row-range mode (tile knob mode = 3; fp32 MatVec-shaped: f = MUL, the second operand the
+// same vector x for every cc point, unit-stride rows of 1024·NV elements): each CTA owns a
+// CONTIGUOUS range of cc points (rows), so the GPU streams ~2 rows per SM at a time through
+// HBM instead of one row per resident warp (thousands of concurrent 32 KB streams), and x
+// is loaded once per thread into registers (thread t holds the 16-byte chunks t + 256·j)
+// instead of once per row.  The next step's rows (8/NV rows: 8 loads per thread) are
+// issued before the current step's rows are folded.  Per row: thread fold in chunk order,
+// warp shuffle tree, warps in order through shared memory (8 rows per barrier) — a fixed
+// association, deterministic.
+template <int NV, int OP>
+__global__ void __launch_bounds__(256, 2) t2_rows_kernel(const __grid_constant__ T2Params P) {
+  __shared__ float red[8][8];
+  const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+  const int64_t G = gridDim.x;
+  const int64_t c0 = P.Ncc * blockIdx.x / G, c1 = P.Ncc * (blockIdx.x + 1) / G;
+  const float4* xb = reinterpret_cast<const float4*>((const float*)P.b + P.bbase) + tid;
+  float4 xv[NV];
+#pragma unroll
+  for (int j = 0; j < NV; ++j) xv[j] = __ldg(xb + 256 * j);
+  auto offs = [&](int64_t c, int64_t* ao, int64_t* oo) {
+    int64_t a = P.abase, o = P.obase, rem = c;
+    for (int t = P.ncc - 1; t >= 0; --t) {
+      const int64_t v = rem % P.ccsize[t];
+      rem /= P.ccsize[t];
+      a += P.aLc[t] * v;
+      o += P.oLc[t] * v;
+    }
+    *ao = a;
+    *oo = o;
+  };
+  auto load = [&](int64_t c, uint4* r) {
+    int64_t ao, oo;
+    offs(c, &ao, &oo);
+    const uint4* pa = reinterpret_cast<const uint4*>((const float*)P.a + ao) + tid;
+#pragma unroll
+    for (int j = 0; j < NV; ++j) r[j] = ld_nc_v4(pa + 256 * j);
+  };
+  // R = 8 / NV rows per step, so every step has 8 16-byte loads per thread in flight
+  constexpr int R = 8 / NV;
+  auto load_step = [&](int64_t s, uint4* r) {
+#pragma unroll
+    for (int q = 0; q < R; ++q)
+      if (s + q < c1) load(s + q, r + q * NV);
+  };
+  uint4 cur[R * NV], nxt[R * NV];
+  if (c0 < c1) load_step(c0, cur);
+  for (int64_t c = c0; c < c1; c += 8) {
+#pragma unroll 1
+    for (int qq = 0; qq < 8; qq += R) {
+      const int64_t s0 = c + qq;
+      if (s0 >= c1) break;                       // CTA-uniform
+      if (s0 + R < c1) load_step(s0 + R, nxt);
+#pragma unroll
+      for (int q = 0; q < R; ++q) {
+        float acc = identity_t<OP, float>();
+#pragma unroll
+        for (int j = 0; j < NV; ++j) {
+          const float* a = reinterpret_cast<const float*>(&cur[q * NV + j]);
+          acc = combine_t<OP, float>(acc, a[0] * xv[j].x);
+          acc = combine_t<OP, float>(acc, a[1] * xv[j].y);
+          acc = combine_t<OP, float>(acc, a[2] * xv[j].z);
+          acc = combine_t<OP, float>(acc, a[3] * xv[j].w);
+        }
+        acc = warp_reduce<OP, float>(acc);
+        if (lane == 0) red[qq + q][warp] = acc;  // rows past c1 are never read
+      }
+#pragma unroll
+      for (int j = 0; j < R * NV; ++j) cur[j] = nxt[j];
+    }
+    __syncthreads();
+    if (tid < 8 && c + tid < c1) {
+      float s = red[tid][0];
+#pragma unroll
+      for (int w = 1; w < 8; ++w) s = combine_t<OP, float>(s, red[tid][w]);
+      int64_t ao, oo;
+      offs(c + tid, &ao, &oo);
+      store_as<float>(P.out, P.odt, oo, s);
+    }
+    __syncthreads();
+  }
+}
+
 template <class TI, class V, int OP, int F>
 __global__ void __launch_bounds__(256) t2_col_kernel(const __grid_constant__ T2Params P) {
   const TI* A = (const TI*)P.a;
@@ -339,10 +421,27 @@ mdh_status prepare_t2(Plan* p) {
     if (p->Ncc < threads) S = (int)std::min<int64_t>(std::max<int64_t>(1, p->Nred / 16), (threads + p->Ncc - 1) / p->Ncc);
   }
   if (p->tiles.split > 0) S = (int)std::min<int64_t>(p->tiles.split, p->Nred);
+  if (p->tiles.mode == 3 && row) S = 1;      // row-range mode: one CTA folds whole rows
   if (S < 1) S = 1;
   p->tiles.split = S;
   // 0 = column mode, 1 = row mode (CTA per unit), 2 = row mode (warp per cc point)
   p->tiles.vec = row ? ((S == 1 && p->Nred <= 65536 && p->Ncc >= 148 * 8) ? 2 : 1) : 0;
+  // 3 = row-range mode (t2_rows_kernel; tile knob mode = 3): fp32 MatVec shape — f = MUL,
+  // one split, unit-stride rows of 1024·{1,2,4,8} elements, the same vector for every row
+  if (p->tiles.mode == 3 && row && S == 1 && p->f == MDH_F_MUL && p->n_in == 2 && p->in[0].dtype == MDH_F32 &&
+      p->in[1].dtype == MDH_F32 && p->compute == MDH_F32) {
+    int64_t bLr = 0;
+    red_linear(*p, p->in[1].acc[0], &bLr);
+    bool ok = bLr == 1 && p->Nred % 1024 == 0 && p->in[0].acc[0].base % 4 == 0 && p->in[1].acc[0].base % 4 == 0;
+    const int64_t nv = p->Nred / 1024;
+    ok = ok && (nv == 1 || nv == 2 || nv == 4 || nv == 8);
+    for (int t = 0; ok && t < p->ncc; ++t)
+      ok = p->in[1].acc[0].L[p->cc[t]] == 0 && p->in[0].acc[0].L[p->cc[t]] % 4 == 0;
+    if (ok) {
+      p->tiles.vec = 3;
+      p->why += " (row-range MatVec kernel)";
+    }
+  }
   size_t part = (S > 1) ? (size_t)p->Ncc * S * compute_size(*p) : 0;
   size_t tick = (S > 1 && row) ? (size_t)p->Ncc * 4 : 0;
   p->ws_kernel = (part + 255) / 256 * 256 + (tick + 255) / 256 * 256;
@@ -354,7 +453,29 @@ static mdh_status launch_typed(const Plan& p, const T2Params& P, cudaStream_t st
   const bool row = p.tiles.vec == 1;
   const int F = p.f;
   int64_t units = P.Ncc * P.S;
-  if (p.tiles.vec == 2) {
+  if constexpr (std::is_same<TI, float>::value) {
+    // row-range mode (tile knob mode = 3): see t2_rows_kernel for the eligibility
+    // (the plan checked the shape; the buffers must be 16-byte aligned, else warp mode)
+    const bool ok = p.tiles.vec == 3 && ((uintptr_t)P.a & 15) == 0 && ((uintptr_t)P.b & 15) == 0;
+    const int64_t nv = P.Nred / 1024;
+    if (ok) {
+      const int per_sm = p.tiles.per_thread >= 2 && p.tiles.per_thread <= 4 ? p.tiles.per_thread : 2;
+      const unsigned g = (unsigned)std::min<int64_t>(P.Ncc, 148LL * per_sm);
+#define T2_ROWS(NV)                                                                               \
+  do {                                                                                            \
+    if (p.redop == MDH_PW_ADD) t2_rows_kernel<NV, MDH_PW_ADD><<<g, 256, 0, st>>>(P);               \
+    else if (p.redop == MDH_PW_MAX) t2_rows_kernel<NV, MDH_PW_MAX><<<g, 256, 0, st>>>(P);          \
+    else t2_rows_kernel<NV, MDH_PW_MIN><<<g, 256, 0, st>>>(P);                                     \
+  } while (0)
+      if (nv == 1) T2_ROWS(1);
+      else if (nv == 2) T2_ROWS(2);
+      else if (nv == 4) T2_ROWS(4);
+      else T2_ROWS(8);
+#undef T2_ROWS
+      return post_launch("t2_rows_kernel");
+    }
+  }
+  if (p.tiles.vec == 2 || p.tiles.vec == 3) {
     unsigned g = (unsigned)std::min<int64_t>((P.Ncc + 7) / 8, 148LL * 16);
 #define T2_WARP(OP, FF) t2_warp_kernel<TI, V, OP, FF><<<g, 256, 0, st>>>(P)
     if (F == MDH_F_MUL) {

@@ -174,6 +174,7 @@ void apply(Tiles* t, const std::string& k, double v) {
   else if (k == "l2pf") t->l2pf = iv;
   else if (k == "nstream") t->nstream = iv;
   else if (k == "areuse") t->areuse = iv;
+  else if (k == "mode") t->mode = iv;
 }
 
 std::string read_file(const char* path) {

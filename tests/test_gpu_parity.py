@@ -73,6 +73,28 @@ def test_matvec(I, K):
     assert_close_full(spec, x, got, 1e-4, kind="rel")
 
 
+@pytest.mark.parametrize("I,K", [(1, 1024), (37, 2048), (1000, 4096), (4096, 4096), (8192, 8192), (300, 8192)])
+@pytest.mark.parametrize("tile", ["mode=3", "mode=3,per_thread=4"])
+def test_matvec_row_range(I, K, tile):
+    """Row-range MatVec kernel (tile knob mode 3: contiguous row ranges per CTA, x held in
+    registers): ragged row ranges (I not a multiple of the grid or of 8), every supported
+    row length, fp32 1e-4 vs the fp64 oracle."""
+    spec = S.matvec(I, K)
+    x = G.gen_inputs(spec, 2150, "positive")
+    got, p = run_gpu(spec, x, force_tile=tile)
+    assert "row-range" in p.describe()["why"], p.describe()["why"]
+    assert_close_full(spec, x, got, 1e-4, kind="rel")
+
+
+@pytest.mark.parametrize("op", ["PW_MAX", "PW_MIN"])
+def test_matvec_row_range_maxmin(op):
+    spec = S.matvec(777, 2048, "f32", op)
+    x = G.gen_inputs(spec, 2160, "signed")
+    got, p = run_gpu(spec, x, force_tile="mode=3")
+    assert "row-range" in p.describe()["why"]
+    assert_close_full(spec, x, got, 1e-6, kind="rel")
+
+
 @pytest.mark.parametrize("op", ["PW_MAX", "PW_MIN", "PW_ADD"])
 def test_matvec_int32(op):
     spec = S.matvec(37, 5001, "i32", op)

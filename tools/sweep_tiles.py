@@ -31,6 +31,8 @@ def cases():
          [f"split={s}" for s in (592, 1184, 2368, 4736)]),
         ("dot_i32_2^20", lambda: (S.dot(1 << 20, "i32"), G.dot_inputs(1 << 20, "i32")),
          [f"split={s}" for s in (64, 128, 148, 256, 296, 512)]),
+        *[(f"matvec_f32_{n}", (lambda n=n: (S.matvec(n, n), G.gen_inputs(S.matvec(n, n), 2100, "positive"))),
+           ["mode=3", "mode=3,per_thread=3"]) for n in (4096, 8192)],
         ("jacobi3d", lambda: (S.jacobi3d(512, 512, 512), G.jacobi3d_inputs(512, 512, 512)),
          [f"zchunk={z}" for z in (8, 16, 32, 64, 128, 255, 510)]),
         ("prl_B", lambda: (S.prl(1 << 14, 1 << 20), G.prl_inputs(1 << 14, 1 << 20)),

@@ -35,6 +35,11 @@ def main():
             Z, Y, X = (int(v) for v in name[4:].split(","))
             w = dict(spec=S.jacobi3d(Z, Y, X), inputs=lambda Z=Z, Y=Y, X=X: G.jacobi3d_inputs(Z, Y, X),
                      work=4.0 * (Z * Y * X + (Z - 2) * (Y - 2) * (X - 2)), unit="GB/s", scale=1e9, bound="hbm", dtype="f32")
+        elif name.startswith("dot:"):         # fp32 Dot of N elements (read-only stream floor)
+            from mdh_workloads import specs as S, gen as G
+            N = int(name[4:])
+            w = dict(spec=S.dot(N, "f32"), inputs=lambda N=N: G.dot_inputs(N, "f32"), work=8.0 * N,
+                     unit="GB/s", scale=1e9, bound="hbm", dtype="f32")
         elif name.startswith("prl:"):         # PRL N new × I DB records
             from mdh_workloads import specs as S, gen as G
             N, I = (int(v) for v in name[4:].split(","))
