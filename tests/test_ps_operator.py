@@ -89,7 +89,8 @@ def test_gpu_prefix_sum(shape, dim, dt):
 @pytest.mark.parametrize("shape,dt,tile", [([3, 200000], "i32", None), ([3, 100003], "f32", None),
                                            ([2, 300001], "f64", "seg=4096"), ([1 << 22], "i64", "seg=65536"),
                                            ([1 << 22], "u32", None), ([5, 65536 * 3 + 4096 * 5 + 1], "f32", None),
-                                           ([(1 << 24) + 12345], "f32", None), ([3, 100003], "f32", "seg=8192")])
+                                           ([(1 << 24) + 12345], "f32", None), ([3, 100003], "f32", "seg=8192"),
+                                           ([(1 << 25) + 3], "f32", None), ([7, 3000017], "i32", None)])
 def test_gpu_single_pass_scan(shape, dt, tile):
     """Long rows take a single-pass scan: the tree scan (default; per-row tree of tile
     aggregates) or the segmented one (tile knob seg): aligned and misaligned row starts,
