@@ -22,6 +22,11 @@ T4_WIDE = ["bn=256", "bn=512", "bn=256,split=1", "bn=512,split=1", "bn=512,stage
 def cases():
     from mdh_workloads import specs as S
     from mdh_workloads import gen as G
+    import bench
+
+    def bw(name):                   # a bench workload's spec and seeded inputs
+        w = bench.workload(name)
+        return w["spec"], w["inputs"]()
     return [
         ("dot_f32_2^20", lambda: (S.dot(1 << 20, "f32"), G.dot_inputs(1 << 20, "f32")),
          [f"split={s}" for s in (64, 128, 148, 256, 296, 512, 592, 1184)]),
@@ -34,7 +39,23 @@ def cases():
         *[(f"matvec_f32_{n}", (lambda n=n: (S.matvec(n, n), G.gen_inputs(S.matvec(n, n), 2100, "positive"))),
            ["mode=3", "mode=3,per_thread=3"]) for n in (4096, 8192)],
         ("jacobi3d", lambda: (S.jacobi3d(512, 512, 512), G.jacobi3d_inputs(512, 512, 512)),
-         [f"zchunk={z}" for z in (8, 16, 32, 64, 128, 255, 510)]),
+         [f"zchunk={z}" for z in (8, 16, 32, 64, 128, 255, 510)]
+         # T1 block shapes (bx threads along x), 8 outputs per thread, L2 prefetch hints, and the
+         # TMA-staged plane ring — every knob of the 7-point kernel
+         + [f"zchunk=8,l2pf=2,per_thread={b}" for b in (64, 128)]
+         + ["zchunk=8,l2pf=2", "zchunk=8,l2pf=1", "zchunk=16,l2pf=2", "zchunk=8,vec=8",
+            "zchunk=8,stages=3", "zchunk=16,stages=6"]),
+        ("gaussian2d", lambda: bw("gaussian2d"),
+         [f"zchunk={z}" for z in (8, 16, 32, 64)]),
+        # T5: records per thread (vec = R), CTAs per SM (stages), DB-loop unroll (bk), split
+        ("prl_A", lambda: bw("prl_A"),
+         ["split=1", "vec=8", "stages=2", "bk=2", "bk=8", "vec=8,bk=2"]),
+        # T3: SGEMM split and the kernel without the register double buffer (stages=1)
+        ("matmul_f32", lambda: bw("matmul_f32"),
+         ["split=1", "split=2", "stages=1"]),
+        # T6: the streaming scan vs the segmented grid-barrier scan at three segment sizes
+        ("prefix_sum_f32", lambda: bw("prefix_sum_f32"),
+         [f"seg={g}" for g in (65536, 262144, 1048576)]),
         ("prl_B", lambda: (S.prl(1 << 14, 1 << 20), G.prl_inputs(1 << 14, 1 << 20)),
          [f"split={s}" for s in (8, 16, 32, 37, 48, 64)]),
         # T4 2-SM: pair-tile width (256 / 512) × whole tiles vs stream-K for the last wave
@@ -118,7 +139,8 @@ def main():
             # the default won: record the knobs it resolved to (a table entry of {} would
             # fall back to the template defaults, not to the nearest bucket it was timed with)
             knobs = {"T1_stencil": ("zchunk", "l2pf"), "T2_reduce": ("split",), "T4_tcgen05_contraction": ("bn", "split", "stages"),
-                     "T5_prl_pairwise": ("split",), "T3_simt_contraction": ("split",)}.get(d["template"], ())
+                     "T5_prl_pairwise": ("split", "vec", "stages", "bk"), "T3_simt_contraction": ("split",),
+                     "T6_prefix_scan": ("seg",)}.get(d["template"], ())
             tiles = {k: int(d["tiles"][k]) for k in knobs if k in d["tiles"]}
         fname = spec["f"]
         opcls = next((o for o in spec["ops"] if o == "PS_ADD"), None) or next((o for o in spec["ops"] if o != "CC"), "CC")
