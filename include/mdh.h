@@ -198,7 +198,18 @@ mdh_status mdh_execute(mdh_plan_t plan, const void* const* in, void* const* out,
 /* End-to-end variant: in/out are HOST pointers (pinned for full PCIe bandwidth).
  * `device_scratch` (>= mdh_plan_host_scratch_size bytes) holds the device copies and
  * the workspace.  Enqueues H2D copies, the computation and D2H copies on the stream;
- * the caller synchronises before reading `out`.                                   */
+ * the caller synchronises before reading `out`.
+ * Pipelined (world-size-1 plans with >= 32 MB of host data, $MDH_HOST_PIPE_MIN_MB; off
+ * with MDH_HOST_PIPE=0): when a cc dim d exists on which every buffer depends only
+ * through its coordinate 0 (MatMul rows, Jacobi planes, MCC images, PRL new records),
+ * the problem runs as 4 chunks along d (virtual shards of the plan): chunk c's input
+ * slices are copied on an internal copy-in stream, computed on `cuda_stream`, and its
+ * output slice copied back on an internal copy-out stream, so both PCIe directions and
+ * the kernels overlap; inputs that do not depend on d are copied once.  The stream
+ * semantics are unchanged: the call's work is ordered after earlier work on
+ * `cuda_stream` and later work on it waits for the last D2H copy.  Host output
+ * elements outside the output image (C-5) are unspecified after the call.
+ * Errors: as mdh_execute; INVALID_ARG for NULL pointers or too little scratch.        */
 mdh_status mdh_plan_host_scratch_size(mdh_plan_t plan, size_t* bytes);
 mdh_status mdh_execute_host(mdh_plan_t plan, const void* const* host_in,
                             void* const* host_out, void* device_scratch,

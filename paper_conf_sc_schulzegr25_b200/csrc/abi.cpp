@@ -8,8 +8,35 @@
 
 #include "internal.h"
 
+#include <mutex>
+#include <vector>
+
+// Pipelined host execution (mdh_execute_host): the problem cut into C chunks along a cc
+// dim on which every buffer depends only through its outermost coordinate, so each chunk's
+// input and output slices are contiguous host ranges.  Chunk c's H2D copies (copy-in
+// stream), its computation (the caller's stream; sub-plan = virtual shard c of C) and its
+// D2H copies (copy-out stream) overlap the neighbouring chunks' — both PCIe directions and
+// the GPU busy at once.
+struct HostPipe {
+  bool built = false, ok = false;
+  int dim = -1, C = 0;
+  std::vector<mdh_plan_t> sub;
+  size_t ws_max = 0;
+  cudaStream_t s_in = nullptr, s_out = nullptr;
+  std::vector<cudaEvent_t> ev;        // [0] entry, [1..C] copied in, [C+1..2C] computed, [2C+1] copied out
+};
+
 struct mdh_plan_s {
   mdh::Plan p;
+  // a copy of the spec and options (world_size 1 plans): the pipeline's sub-plans
+  bool have_spec = false;
+  mdh_spec spec{};
+  std::vector<mdh_buffer> sin, sout;
+  std::vector<double> fpar;
+  mdh_plan_opts opts{};
+  std::string tile_table, force_tile;
+  std::mutex mu;
+  HostPipe pipe;
 };
 
 namespace mdh {
@@ -165,6 +192,172 @@ static mdh_status execute_sharded(const mdh::Plan& p, const void* const* in, voi
 
 }  // namespace mdh
 
+// Build the pipeline of a world-size-1 plan once (under h->mu): the first cc dim d on which
+// every input and output buffer depends only through its coordinate 0 (or not at all),
+// every output depending on it; C = 4 chunks as virtual shards of the plan on d.  Not
+// built (ok = false) for small problems (< 32 MB of host data), when no dim qualifies, or
+// with MDH_HOST_PIPE=0.
+static void build_pipe(mdh_plan_s* h) {
+  HostPipe& P = h->pipe;
+  P.built = true;
+  const mdh::Plan& p = h->p;
+  if (!h->have_spec || p.world > 1 || p.sharded) return;
+  const char* env = std::getenv("MDH_HOST_PIPE");
+  if (env && env[0] == '0') return;
+  size_t bytes = 0;
+  for (int b = 0; b < p.n_in; ++b) bytes += (size_t)p.in[b].elems * mdh::dtype_size(p.in[b].dtype);
+  for (int b = 0; b < p.n_out; ++b) bytes += (size_t)p.out[b].elems * mdh::dtype_size(p.out[b].dtype);
+  const char* mn = std::getenv("MDH_HOST_PIPE_MIN_MB");      // (tests: pipeline small problems)
+  if (bytes < ((size_t)(mn ? std::atoi(mn) : 32) << 20)) return;
+  const mdh_spec& sp = h->spec;
+  for (int d = 0; d < sp.D && !P.ok; ++d) {
+    if (sp.op[d] != MDH_CC || sp.size[d] < 4) continue;
+    bool ok = true;
+    auto dep = [&](const mdh_buffer& B, bool* any) {
+      *any = false;
+      for (int a = 0; a < B.n_acc; ++a)
+        for (int r = 0; r < B.rank; ++r)
+          if (B.acc[a].coeff[r][d] != 0) {
+            if (r != 0) ok = false;
+            *any = true;
+          }
+    };
+    bool any;
+    for (int b = 0; b < sp.n_in; ++b) dep(sp.in[b], &any);
+    for (int b = 0; b < sp.n_out; ++b) {
+      dep(sp.out[b], &any);
+      ok = ok && any;
+    }
+    if (!ok) continue;
+    const int C = (int)std::min<int64_t>(4, sp.size[d]);
+    std::vector<mdh_plan_t> sub(C, nullptr);
+    size_t wsm = p.ws_total;
+    for (int c = 0; c < C && ok; ++c) {
+      mdh_plan_opts o = h->opts;
+      o.world_size = C;
+      o.rank = c;
+      o.shard_dim = d;
+      o.nccl_comm = nullptr;
+      o.flags |= MDH_PLAN_VIRTUAL_SHARD;
+      if (mdh_plan(&sp, &o, &sub[c]) != MDH_OK) {
+        ok = false;
+        break;
+      }
+      const mdh::Plan& q = sub[c]->p;
+      wsm = std::max(wsm, q.ws_total);
+      // slices must be contiguous: only coordinate 0 cut
+      auto contiguous = [&](const mdh::Buf& L, const mdh::Buf& F) {
+        for (int r = 1; r < F.rank; ++r)
+          if (L.goff[r] != 0 || L.shape[r] != F.shape[r]) return false;
+        return true;
+      };
+      for (int b = 0; b < p.n_in && ok; ++b) ok = contiguous(q.in[b], p.in[b]);
+      for (int b = 0; b < p.n_out && ok; ++b) ok = contiguous(q.out[b], p.out[b]);
+    }
+    if (ok) {
+      ok = cudaStreamCreateWithFlags(&P.s_in, cudaStreamNonBlocking) == cudaSuccess &&
+           cudaStreamCreateWithFlags(&P.s_out, cudaStreamNonBlocking) == cudaSuccess;
+      P.ev.assign(2 * C + 2, nullptr);
+      for (auto& e : P.ev) ok = ok && cudaEventCreateWithFlags(&e, cudaEventDisableTiming) == cudaSuccess;
+    }
+    if (!ok) {
+      for (auto q : sub) mdh_destroy(q);
+      cudaGetLastError();
+      continue;
+    }
+    P.ok = true;
+    P.dim = d;
+    P.C = C;
+    P.sub = sub;
+    P.ws_max = wsm;
+  }
+}
+
+static void ensure_pipe(mdh_plan_s* h) {
+  std::lock_guard<std::mutex> g(h->mu);
+  if (!h->pipe.built) build_pipe(h);
+}
+
+static size_t host_bytes(const mdh::Buf& B) { return (size_t)B.elems * mdh::dtype_size(B.dtype); }
+
+// elements of buffer F (full shape) before the slice L (coordinate 0 from goff[0]) and in it
+static void slice_of(const mdh::Buf& L, const mdh::Buf& F, size_t* off, size_t* n) {
+  size_t row = 1;
+  for (int r = 1; r < F.rank; ++r) row *= (size_t)F.shape[r];
+  size_t e = 1;
+  for (int r = 0; r < L.rank; ++r) e *= (size_t)L.shape[r];
+  *off = (size_t)L.goff[0] * row;
+  *n = e;
+}
+
+// the pipelined mdh_execute_host (HostPipe); returns UNSUPPORTED (nothing enqueued) when a
+// chunk pointer would be misaligned, so the caller takes the one-shot path
+static mdh_status execute_host_pipe(mdh_plan_s* h, const void* const* host_in, void* const* host_out, char* base,
+                                    cudaStream_t st) {
+  const mdh::Plan& p = h->p;
+  HostPipe& P = h->pipe;
+  const int C = P.C;
+  std::vector<char*> din(p.n_in), dout(p.n_out);
+  size_t off = 0;
+  for (int b = 0; b < p.n_in; ++b) { din[b] = base + off; off += (host_bytes(p.in[b]) + 255) / 256 * 256; }
+  for (int b = 0; b < p.n_out; ++b) { dout[b] = base + off; off += (host_bytes(p.out[b]) + 255) / 256 * 256; }
+  char* ws = base + off;
+  // chunk slices (element offset, count) and the alignment the kernels need
+  std::vector<size_t> io(C * p.n_in), in_n(C * p.n_in), oo(C * p.n_out), on(C * p.n_out);
+  std::vector<bool> shared(p.n_in, true);
+  for (int c = 0; c < C; ++c) {
+    const mdh::Plan& q = P.sub[c]->p;
+    for (int b = 0; b < p.n_in; ++b) {
+      slice_of(q.in[b], p.in[b], &io[c * p.n_in + b], &in_n[c * p.n_in + b]);
+      if (in_n[c * p.n_in + b] != (size_t)p.in[b].elems) shared[b] = false;
+      if ((io[c * p.n_in + b] * mdh::dtype_size(p.in[b].dtype)) % 16) return MDH_ERR_UNSUPPORTED;
+    }
+    for (int b = 0; b < p.n_out; ++b) {
+      slice_of(q.out[b], p.out[b], &oo[c * p.n_out + b], &on[c * p.n_out + b]);
+      if ((oo[c * p.n_out + b] * mdh::dtype_size(p.out[b].dtype)) % 16) return MDH_ERR_UNSUPPORTED;
+    }
+  }
+  MDH_CUDA(cudaEventRecord(P.ev[0], st));
+  MDH_CUDA(cudaStreamWaitEvent(P.s_in, P.ev[0], 0));
+  MDH_CUDA(cudaStreamWaitEvent(P.s_out, P.ev[0], 0));
+  for (int b = 0; b < p.n_in; ++b)                    // inputs every chunk reads whole: once
+    if (shared[b]) MDH_CUDA(cudaMemcpyAsync(din[b], host_in[b], host_bytes(p.in[b]), cudaMemcpyHostToDevice, P.s_in));
+  for (int c = 0; c < C; ++c) {
+    for (int b = 0; b < p.n_in; ++b) {
+      if (shared[b]) continue;
+      const size_t es = mdh::dtype_size(p.in[b].dtype), o = io[c * p.n_in + b] * es;
+      MDH_CUDA(cudaMemcpyAsync(din[b] + o, (const char*)host_in[b] + o, in_n[c * p.n_in + b] * es,
+                               cudaMemcpyHostToDevice, P.s_in));
+    }
+    MDH_CUDA(cudaEventRecord(P.ev[1 + c], P.s_in));
+  }
+  if (P.ws_max) MDH_CUDA(cudaMemsetAsync(ws, 0, P.ws_max, st));   // workspace contract
+  int launched = 0;
+  for (int c = 0; c < C; ++c) {
+    MDH_CUDA(cudaStreamWaitEvent(st, P.ev[1 + c], 0));
+    const void* ci[MDH_MAX_BUFS];
+    void* co[MDH_MAX_BUFS];
+    for (int b = 0; b < p.n_in; ++b) ci[b] = din[b] + io[c * p.n_in + b] * mdh::dtype_size(p.in[b].dtype);
+    for (int b = 0; b < p.n_out; ++b) co[b] = dout[b] + oo[c * p.n_out + b] * mdh::dtype_size(p.out[b].dtype);
+    MDH_TRY(mdh_execute(P.sub[c], ci, co, ws, P.ws_max, st));
+    launched += mdh::launch_count();
+    MDH_CUDA(cudaEventRecord(P.ev[1 + C + c], st));
+  }
+  for (int c = 0; c < C; ++c) {
+    MDH_CUDA(cudaStreamWaitEvent(P.s_out, P.ev[1 + C + c], 0));
+    for (int b = 0; b < p.n_out; ++b) {
+      const size_t es = mdh::dtype_size(p.out[b].dtype), o = oo[c * p.n_out + b] * es;
+      MDH_CUDA(cudaMemcpyAsync((char*)host_out[b] + o, dout[b] + o, on[c * p.n_out + b] * es, cudaMemcpyDeviceToHost,
+                               P.s_out));
+    }
+  }
+  MDH_CUDA(cudaEventRecord(P.ev[2 * C + 1], P.s_out));
+  MDH_CUDA(cudaStreamWaitEvent(st, P.ev[2 * C + 1], 0));
+  mdh::reset_launch_count();
+  mdh::count_launch(launched);
+  return MDH_OK;
+}
+
 using mdh::set_error;
 
 extern "C" {
@@ -184,6 +377,22 @@ mdh_status mdh_plan(const mdh_spec* spec, const mdh_plan_opts* opts, mdh_plan_t*
   if (s != MDH_OK) {
     mdh_destroy(h);
     return s;
+  }
+  if (spec && (!opts || opts->world_size <= 1) && !h->p.sharded) {
+    h->sin.assign(spec->in, spec->in + spec->n_in);
+    h->sout.assign(spec->out, spec->out + spec->n_out);
+    if (spec->fparams && spec->n_fparams > 0) h->fpar.assign(spec->fparams, spec->fparams + spec->n_fparams);
+    h->spec = *spec;
+    h->spec.in = h->sin.data();
+    h->spec.out = h->sout.data();
+    h->spec.fparams = h->fpar.empty() ? nullptr : h->fpar.data();
+    if (opts) h->opts = *opts;
+    else h->opts.world_size = 1, h->opts.shard_dim = -1;
+    if (h->opts.tile_table) h->tile_table = h->opts.tile_table;
+    if (h->opts.force_tile) h->force_tile = h->opts.force_tile;
+    h->opts.tile_table = h->tile_table.empty() ? nullptr : h->tile_table.c_str();
+    h->opts.force_tile = h->force_tile.empty() ? nullptr : h->force_tile.c_str();
+    h->have_spec = true;
   }
   *plan_out = h;
   return MDH_OK;
@@ -214,6 +423,11 @@ mdh_status mdh_plan_local_shape(mdh_plan_t plan, int32_t is_output, int32_t buf,
 mdh_status mdh_plan_describe(mdh_plan_t plan, char* json, size_t cap, size_t* needed) {
   if (!plan) { set_error("NULL plan"); return MDH_ERR_INVALID_ARG; }
   std::string s = mdh::describe_plan(plan->p);
+  if (plan->pipe.ok && !s.empty() && s.back() == '}') {    // the mdh_execute_host pipeline, once built
+    s.pop_back();
+    s += ", \"host_pipe\": {\"dim\": " + std::to_string(plan->pipe.dim) + ", \"chunks\": " +
+         std::to_string(plan->pipe.C) + "}}";
+  }
   if (needed) *needed = s.size() + 1;
   if (json && cap > 0) {
     size_t n = std::min(cap - 1, s.size());
@@ -254,7 +468,8 @@ mdh_status mdh_plan_host_scratch_size(mdh_plan_t plan, size_t* bytes) {
   size_t s = 0;
   for (int b = 0; b < p.n_in; ++b) s += ((size_t)p.in[b].elems * mdh::dtype_size(p.in[b].dtype) + 255) / 256 * 256;
   for (int b = 0; b < p.n_out; ++b) s += ((size_t)p.out[b].elems * mdh::dtype_size(p.out[b].dtype) + 255) / 256 * 256;
-  *bytes = s + p.ws_total + 256;
+  ensure_pipe(plan);
+  *bytes = s + std::max(p.ws_total, plan->pipe.ok ? plan->pipe.ws_max : (size_t)0) + 256;
   return MDH_OK;
 }
 
@@ -267,6 +482,10 @@ mdh_status mdh_execute_host(mdh_plan_t plan, const void* const* host_in, void* c
   if (scratch_bytes < need) { set_error("device scratch of %zu bytes < %zu needed", scratch_bytes, need); return MDH_ERR_INVALID_ARG; }
   cudaStream_t st = (cudaStream_t)cuda_stream;
   char* base = (char*)(((uintptr_t)device_scratch + 255) / 256 * 256);
+  if (plan->pipe.ok) {                       // chunked: copies in both directions overlap the kernels
+    const mdh_status ps = execute_host_pipe(plan, host_in, host_out, base, st);
+    if (ps != MDH_ERR_UNSUPPORTED) return ps;
+  }
   const void* din[MDH_MAX_BUFS];
   void* dout[MDH_MAX_BUFS];
   size_t off = 0;
@@ -420,6 +639,11 @@ mdh_status mdh_destroy(mdh_plan_t plan) {
     cudaSetDevice(cur);
   }
   mdh::release_t4(&plan->p);
+  for (auto q : plan->pipe.sub) mdh_destroy(q);
+  for (auto e : plan->pipe.ev)
+    if (e) cudaEventDestroy(e);
+  if (plan->pipe.s_in) cudaStreamDestroy(plan->pipe.s_in);
+  if (plan->pipe.s_out) cudaStreamDestroy(plan->pipe.s_out);
   delete plan;
   return MDH_OK;
 }
