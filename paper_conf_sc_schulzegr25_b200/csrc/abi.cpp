@@ -254,11 +254,15 @@ static void build_pipe(mdh_plan_s* h) {
       for (int b = 0; b < p.n_in && ok; ++b) ok = contiguous(q.in[b], p.in[b]);
       for (int b = 0; b < p.n_out && ok; ++b) ok = contiguous(q.out[b], p.out[b]);
     }
-    if (ok) {
+    if (ok) {                           // the copy streams and events live on the plan's device
+      int cur = 0;
+      cudaGetDevice(&cur);
+      cudaSetDevice(p.device);
       ok = cudaStreamCreateWithFlags(&P.s_in, cudaStreamNonBlocking) == cudaSuccess &&
            cudaStreamCreateWithFlags(&P.s_out, cudaStreamNonBlocking) == cudaSuccess;
       P.ev.assign(2 * C + 2, nullptr);
       for (auto& e : P.ev) ok = ok && cudaEventCreateWithFlags(&e, cudaEventDisableTiming) == cudaSuccess;
+      cudaSetDevice(cur);
     }
     if (!ok) {
       for (auto q : sub) mdh_destroy(q);
@@ -483,6 +487,7 @@ mdh_status mdh_execute_host(mdh_plan_t plan, const void* const* host_in, void* c
   cudaStream_t st = (cudaStream_t)cuda_stream;
   char* base = (char*)(((uintptr_t)device_scratch + 255) / 256 * 256);
   if (plan->pipe.ok) {                       // chunked: copies in both directions overlap the kernels
+    std::lock_guard<std::mutex> g(plan->mu);  // (the plan's copy streams and events)
     const mdh_status ps = execute_host_pipe(plan, host_in, host_out, base, st);
     if (ps != MDH_ERR_UNSUPPORTED) return ps;
   }
