@@ -158,7 +158,21 @@ struct T3Lin {
 // FP (fragment-pipelined) = true: one CTA per SM (up to 255 registers) and the shared-memory
 // fragments of k-step kk+1 loaded into a second register set while the 64 FMAs of k-step kk
 // run (no short-scoreboard stall on the LDS results)
-template <bool FP>
+// FFMA2 (sm_100 `fma.rn.f32x2`; default, tile knob mode=0: FFMA): the 8×8 accumulators as 32 fp32 pairs,
+// acc[i][2j..2j+1] = fma(a_i, b[2j..2j+1], acc) in one instruction — the same per-element
+// fp32 FMA sequence (bit-identical results), half the FMA instructions to issue
+__device__ __forceinline__ void ffma2(unsigned long long& acc, unsigned long long a2, unsigned long long b2) {
+  asm("fma.rn.f32x2 %0, %1, %2, %0;" : "+l"(acc) : "l"(a2), "l"(b2));
+}
+__device__ __forceinline__ unsigned long long pair2(float x, float y) {
+  unsigned long long r;
+  asm("mov.b64 %0, {%1, %2};" : "=l"(r) : "f"(x), "f"(y));
+  return r;
+}
+__device__ __forceinline__ float lo2(unsigned long long v) { return __uint_as_float((unsigned)v); }
+__device__ __forceinline__ float hi2(unsigned long long v) { return __uint_as_float((unsigned)(v >> 32)); }
+
+template <bool FP, bool F2 = false>
 __global__ void __launch_bounds__(256, FP ? 1 : 2) t3_linear_kernel(const __grid_constant__ T3Lin P) {
   constexpr int KB = FP ? 16 : 8;                 // k-block (FP: half as many barriers)
   constexpr int H = KB / 8;                        // 8-deep slices per k-block
@@ -208,10 +222,15 @@ __global__ void __launch_bounds__(256, FP ? 1 : 2) t3_linear_kernel(const __grid
     }
   };
   float acc[8][8];
+  unsigned long long acc2[8][4];           // (F2) acc[i][2j], acc[i][2j+1]
 #pragma unroll
   for (int i = 0; i < 8; ++i)
 #pragma unroll
     for (int j = 0; j < 8; ++j) acc[i][j] = 0.f;
+#pragma unroll
+  for (int i = 0; i < 8; ++i)
+#pragma unroll
+    for (int j = 0; j < 4; ++j) acc2[i][j] = 0ull;
   gload(0);
   sstore(0);
   __syncthreads();
@@ -238,10 +257,22 @@ __global__ void __launch_bounds__(256, FP ? 1 : 2) t3_linear_kernel(const __grid
                             fa[cur][1].x, fa[cur][1].y, fa[cur][1].z, fa[cur][1].w};
         const float b[8] = {fb[cur][0].x, fb[cur][0].y, fb[cur][0].z, fb[cur][0].w,
                             fb[cur][1].x, fb[cur][1].y, fb[cur][1].z, fb[cur][1].w};
+        if (F2) {
+          unsigned long long b2[4];
 #pragma unroll
-        for (int i = 0; i < 8; ++i)
+          for (int j = 0; j < 4; ++j) b2[j] = pair2(b[2 * j], b[2 * j + 1]);
 #pragma unroll
-          for (int j = 0; j < 8; ++j) acc[i][j] = fmaf(a[i], b[j], acc[i][j]);
+          for (int i = 0; i < 8; ++i) {
+            const unsigned long long a2 = pair2(a[i], a[i]);
+#pragma unroll
+            for (int j = 0; j < 4; ++j) ffma2(acc2[i][j], a2, b2[j]);
+          }
+        } else {
+#pragma unroll
+          for (int i = 0; i < 8; ++i)
+#pragma unroll
+            for (int j = 0; j < 8; ++j) acc[i][j] = fmaf(a[i], b[j], acc[i][j]);
+        }
       }
     } else {
 #pragma unroll
@@ -263,6 +294,15 @@ __global__ void __launch_bounds__(256, FP ? 1 : 2) t3_linear_kernel(const __grid
       __syncthreads();
       buf ^= 1;
     }
+  }
+  if (F2) {
+#pragma unroll
+    for (int i = 0; i < 8; ++i)
+#pragma unroll
+      for (int j = 0; j < 4; ++j) {
+        acc[i][2 * j] = lo2(acc2[i][j]);
+        acc[i][2 * j + 1] = hi2(acc2[i][j]);
+      }
   }
 #pragma unroll
   for (int i = 0; i < 8; ++i) {
@@ -414,7 +454,9 @@ mdh_status launch_t3(const Plan& p, const void* const* in, void* const* out, voi
     // default: the fragment-pipelined one-CTA-per-SM variant with 16-deep k-blocks (MatMul
     // 4096³ fp32 2.94 ms, 63 % of FFMA; 3.05 ms with 8-deep k-blocks; 3.80 ms for two
     // 128-register CTAs per SM); tile knob stages=1 selects the latter
+    // FFMA2 pairs by default (2.895 vs 2.936 ms, bit-identical); tile knob mode=0 the FFMA form
     if (p.tiles.stages == 1) t3_linear_kernel<false><<<grid, 256, 0, st>>>(L);
+    else if (p.tiles.mode != 0) t3_linear_kernel<true, true><<<grid, 256, 0, st>>>(L);
     else t3_linear_kernel<true><<<grid, 256, 0, st>>>(L);
     return post_launch("t3_linear_kernel");
   }

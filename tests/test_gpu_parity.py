@@ -215,6 +215,21 @@ def test_matmul_fp32(mnk):
     assert_close_full(spec, x, got, 1e-4, kind="rel")
 
 
+@pytest.mark.parametrize("mnk", [(3, 5, 7), (127, 129, 65), (128, 256, 64), (300, 200, 1000), (1000, 777, 333)])
+def test_matmul_fp32_ffma2(mnk):
+    """T3 SGEMM with the accumulators as fp32 pairs (FFMA2, the default; tile knob mode=0 the
+    FFMA form): the same fp32 FMA sequence per element — bit-identical — and 1e-4 of the
+    oracle."""
+    M, N, K = mnk
+    spec = S.matmul(M, N, K)
+    x = G.matmul_inputs(M, N, K, "f32", "signed")
+    got, p = run_gpu(spec, x, force_tile="mode=1")
+    ref, _ = run_gpu(spec, x, force_tile="mode=0")
+    assert p.template == "T3_simt_contraction"
+    assert np.array_equal(got[0], ref[0])
+    assert_close_full(spec, x, got, 1e-4, kind="scale")
+
+
 def test_matmul_fp32_full_size_sampled():
     spec = S.matmul(4096, 4096, 4096)
     x = G.matmul_inputs(4096, 4096, 4096, "f32", "signed")
