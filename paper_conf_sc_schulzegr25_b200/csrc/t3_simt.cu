@@ -158,7 +158,9 @@ struct T3Lin {
 // FP (fragment-pipelined) = true: one CTA per SM (up to 255 registers) and the shared-memory
 // fragments of k-step kk+1 loaded into a second register set while the 64 FMAs of k-step kk
 // run (no short-scoreboard stall on the LDS results)
-// FFMA2 (sm_100 `fma.rn.f32x2`; default, tile knob mode=0: FFMA): the 8×8 accumulators as 32 fp32 pairs,
+// FFMA2 (sm_100 `fma.rn.f32x2`; default, tile knob mode=0: FFMA): the 8×8 accumulators as 32 fp32 pairs
+// (32 instead of 64 FMA instructions per k-step, and 126 registers without spills, so two
+// CTAs fit an SM),
 // acc[i][2j..2j+1] = fma(a_i, b[2j..2j+1], acc) in one instruction — the same per-element
 // fp32 FMA sequence (bit-identical results), half the FMA instructions to issue
 __device__ __forceinline__ void ffma2(unsigned long long& acc, unsigned long long a2, unsigned long long b2) {
@@ -283,10 +285,22 @@ __global__ void __launch_bounds__(256, FP ? 1 : 2) t3_linear_kernel(const __grid
       const float4 b1 = *reinterpret_cast<const float4*>(&Bs[buf][kk][64 + tx * 4]);
       const float a[8] = {a0.x, a0.y, a0.z, a0.w, a1.x, a1.y, a1.z, a1.w};
       const float b[8] = {b0.x, b0.y, b0.z, b0.w, b1.x, b1.y, b1.z, b1.w};
+      if (F2) {
+        unsigned long long b2[4];
 #pragma unroll
-      for (int i = 0; i < 8; ++i)
+        for (int j = 0; j < 4; ++j) b2[j] = pair2(b[2 * j], b[2 * j + 1]);
 #pragma unroll
-        for (int j = 0; j < 8; ++j) acc[i][j] = fmaf(a[i], b[j], acc[i][j]);
+        for (int i = 0; i < 8; ++i) {
+          const unsigned long long a2 = pair2(a[i], a[i]);
+#pragma unroll
+          for (int j = 0; j < 4; ++j) ffma2(acc2[i][j], a2, b2[j]);
+        }
+      } else {
+#pragma unroll
+        for (int i = 0; i < 8; ++i)
+#pragma unroll
+          for (int j = 0; j < 8; ++j) acc[i][j] = fmaf(a[i], b[j], acc[i][j]);
+      }
     }
     }
     if (more) {
@@ -451,13 +465,19 @@ mdh_status launch_t3(const Plan& p, const void* const* in, void* const* out, voi
     L.ldc = (int)p.auxi[3];
     dim3 grid((unsigned)((c.N + 127) / 128), (unsigned)((c.M + 127) / 128));
     if (grid.y > 65535) { set_error("T3: grid too large"); return MDH_ERR_UNSUPPORTED; }
-    // default: the fragment-pipelined one-CTA-per-SM variant with 16-deep k-blocks (MatMul
-    // 4096³ fp32 2.94 ms, 63 % of FFMA; 3.05 ms with 8-deep k-blocks; 3.80 ms for two
-    // 128-register CTAs per SM); tile knob stages=1 selects the latter
-    // FFMA2 pairs by default (2.895 vs 2.936 ms, bit-identical); tile knob mode=0 the FFMA form
-    if (p.tiles.stages == 1) t3_linear_kernel<false><<<grid, 256, 0, st>>>(L);
-    else if (p.tiles.mode != 0) t3_linear_kernel<true, true><<<grid, 256, 0, st>>>(L);
-    else t3_linear_kernel<true><<<grid, 256, 0, st>>>(L);
+    // default: two 128-register CTAs per SM, 8-deep k-blocks, accumulators as FFMA2 pairs
+    // (MatMul 4096³ fp32 2.694 ms = 0.71 of the measured FFMA peak; with FFMA 3.795 ms — it
+    // spilled); tile knob stages=2: one CTA per SM with 16-deep k-blocks and the next
+    // k-step's fragments prefetched into a second register set (2.897 / FFMA 2.936 ms);
+    // tile knob mode=0: the FFMA form of either
+    const bool f2 = p.tiles.mode != 0;
+    if (p.tiles.stages == 2) {
+      if (f2) t3_linear_kernel<true, true><<<grid, 256, 0, st>>>(L);
+      else t3_linear_kernel<true><<<grid, 256, 0, st>>>(L);
+    } else {
+      if (f2) t3_linear_kernel<false, true><<<grid, 256, 0, st>>>(L);
+      else t3_linear_kernel<false><<<grid, 256, 0, st>>>(L);
+    }
     return post_launch("t3_linear_kernel");
   }
   const char* dc = nullptr;

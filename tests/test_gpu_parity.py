@@ -223,11 +223,12 @@ def test_matmul_fp32_ffma2(mnk):
     M, N, K = mnk
     spec = S.matmul(M, N, K)
     x = G.matmul_inputs(M, N, K, "f32", "signed")
-    got, p = run_gpu(spec, x, force_tile="mode=1")
-    ref, _ = run_gpu(spec, x, force_tile="mode=0")
-    assert p.template == "T3_simt_contraction"
-    assert np.array_equal(got[0], ref[0])
-    assert_close_full(spec, x, got, 1e-4, kind="scale")
+    for st in ("stages=4", "stages=2"):       # two CTAs per SM (default) / fragment-pipelined
+        got, p = run_gpu(spec, x, force_tile=st + ",mode=1")
+        ref, _ = run_gpu(spec, x, force_tile=st + ",mode=0")
+        assert p.template == "T3_simt_contraction"
+        assert np.array_equal(got[0], ref[0])
+        assert_close_full(spec, x, got, 1e-4, kind="scale")
 
 
 def test_matmul_fp32_full_size_sampled():

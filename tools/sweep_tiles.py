@@ -50,9 +50,9 @@ def cases():
         # T5: records per thread (vec = R), CTAs per SM (stages), DB-loop unroll (bk), split
         ("prl_A", lambda: bw("prl_A"),
          ["split=1", "vec=8", "stages=2", "bk=2", "bk=8", "vec=8,bk=2"]),
-        # T3: SGEMM split and the kernel without the register double buffer (stages=1)
+        # T3: SGEMM split, the one-CTA-per-SM fragment-pipelined kernel (stages=2), the FFMA form (mode=0)
         ("matmul_f32", lambda: bw("matmul_f32"),
-         ["split=1", "split=2", "stages=1"]),
+         ["split=1", "split=2", "stages=2", "mode=0", "stages=2,mode=0"]),
         # T6: the streaming scan vs the segmented grid-barrier scan at three segment sizes
         ("prefix_sum_f32", lambda: bw("prefix_sum_f32"),
          [f"seg={g}" for g in (65536, 262144, 1048576)]),
