@@ -187,3 +187,15 @@ def test_sweeps_argument_checks_on_host(mdh):
     assert call(base, base + 2 * n, sweeps=2, halo=h) == INVALID_ARG   # peer: one sweep per call
     h.peer_hi[1] = base + n                                      # a "peer" plane inside own v
     assert call(base, base + n, sweeps=1, halo=h) == INVALID_ARG
+
+
+def test_tile_table_picks_the_matvec_row_range_mode(mdh):
+    """The measured tile table (compiled in) selects T2's row-range kernel for MatVec 8192²
+    and keeps warp mode for 4096² (tools/sweep_tiles.py, profiles/r2_matvec_jacobi_floor.txt);
+    a forced mode=3 on a shape it cannot serve (row length not 1024·2^k) stays in warp mode."""
+    d = mdh.Plan(S.matvec(8192, 8192)).describe()
+    assert d["tiles"]["mode"] == 3 and "row-range" in d["why"], d
+    d = mdh.Plan(S.matvec(4096, 4096)).describe()
+    assert d["tiles"]["mode"] != 3 and "row-range" not in d["why"], d
+    d = mdh.Plan(S.matvec(8192, 5000), force_tile="mode=3").describe()
+    assert "row-range" not in d["why"], d
