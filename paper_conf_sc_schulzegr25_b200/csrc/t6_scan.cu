@@ -996,8 +996,7 @@ mdh_status prepare_t6(Plan* p) {
 template <class V>
 static mdh_status launch_seg(const T6Params& P0, char* ws, cudaStream_t st) {
   T6Params P = P0;
-  static int occ[8] = {0};               // resident CTAs per SM, per value size (cached)
-  int& o = occ[sizeof(V)];
+  static int o = 0;                      // resident CTAs per SM (cached per instantiation)
   if (o == 0) {
     MDH_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&o, t6_seg_scan_kernel<V>, T6S_THREADS, 0));
     o = std::max(1, std::min(o, 8));
@@ -1015,13 +1014,15 @@ static mdh_status launch_seg(const T6Params& P0, char* ws, cudaStream_t st) {
 
 template <class V>
 static mdh_status launch_stream(T6Params& P, cudaStream_t st) {
-  static std::once_flag once[8];
-  static cudaError_t aerr[8];
-  std::call_once(once[sizeof(V)], [] {
-    aerr[sizeof(V)] = cudaFuncSetAttribute((const void*)t6_stream_scan_kernel<V>,
-                                           cudaFuncAttributeMaxDynamicSharedMemorySize, t6_smem<V>());
+  // one attribute call per instantiation (a function-local static of the template: V = 4-
+  // and 8-byte types each get their own; indexing a shared array by sizeof(V) overran it)
+  static std::once_flag once;
+  static cudaError_t aerr = cudaSuccess;
+  std::call_once(once, [] {
+    aerr = cudaFuncSetAttribute((const void*)t6_stream_scan_kernel<V>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                t6_smem<V>());
   });
-  MDH_CUDA(aerr[sizeof(V)]);
+  MDH_CUDA(aerr);
   int dev = 0, sms = 148;
   MDH_CUDA(cudaGetDevice(&dev));
   MDH_CUDA(cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev));
