@@ -200,7 +200,8 @@ mdh_status mdh_execute(mdh_plan_t plan, const void* const* in, void* const* out,
  * the workspace.  Enqueues H2D copies, the computation and D2H copies on the stream;
  * the caller synchronises before reading `out`.
  * Pipelined (world-size-1 plans with >= 32 MB of host data, $MDH_HOST_PIPE_MIN_MB; off
- * with MDH_HOST_PIPE=0): when a cc dim d exists on which every buffer depends only
+ * with MDH_HOST_PIPE=0; $MDH_HOST_PIPE_CHUNKS chunks, default 4 — MatMul 4096³ e2e
+ * 66.2 / 67.2 / 65.7 TFLOP/s at 4 / 8 / 16): when a cc dim d exists on which every buffer depends only
  * through its coordinate 0 (MatMul rows, Jacobi planes, MCC images, PRL new records),
  * the problem runs as 4 chunks along d (virtual shards of the plan): chunk c's input
  * slices are copied on an internal copy-in stream, computed on `cuda_stream`, and its

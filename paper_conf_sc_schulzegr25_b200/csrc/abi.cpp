@@ -229,7 +229,8 @@ static void build_pipe(mdh_plan_s* h) {
       ok = ok && any;
     }
     if (!ok) continue;
-    const int C = (int)std::min<int64_t>(4, sp.size[d]);
+    const char* ce = std::getenv("MDH_HOST_PIPE_CHUNKS");
+    const int C = (int)std::min<int64_t>(ce ? std::max(2, std::atoi(ce)) : 4, sp.size[d]);
     std::vector<mdh_plan_t> sub(C, nullptr);
     size_t wsm = p.ws_total;
     for (int c = 0; c < C && ok; ++c) {
