@@ -75,7 +75,7 @@ def cases():
            T4_WIDE + ["bn=256,split=2", "bn=512,split=2", "bn=512,split=2,stages=3"])
           for m in (2048, 1024, 512)],
         *[(f"rank_jacobi3d_{z}", (lambda z=z: (S.jacobi3d(z, 512, 512), G.jacobi3d_inputs(z, 512, 512))),
-           [f"zchunk={c}" for c in (4, 8, 16, 32)]) for z in (257, 130, 66)],
+           [f"zchunk={c},l2pf=2" for c in (3, 4, 5, 6, 7, 8, 10, 12, 16, 32)]) for z in (257, 130, 66)],
         *[(f"rank_prl_A_{i}", (lambda i=i: (S.prl(1 << 20, i), G.prl_inputs(1 << 20, i))),
            [f"split={c}" for c in (1, 2, 3, 4)]) for i in (8192, 4096, 2048)],
         *[(f"rank_prl_B_{i}", (lambda i=i: (S.prl(1 << 14, i), G.prl_inputs(1 << 14, i))),
