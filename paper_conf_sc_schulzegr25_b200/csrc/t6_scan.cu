@@ -1186,6 +1186,7 @@ mdh_status launch_t6(const Plan& p, const void* const* in, void* const* out, voi
       // splits so that the blocks fill 8 × 256 threads per SM, rows per thread ≥ 32
       int64_t S = std::max<int64_t>(1, (int64_t)sms * 8 / std::max<int64_t>(1, groups));
       S = std::min<int64_t>({S, (int64_t)T6_COL_SMAX, std::max<int64_t>(1, P.pwsize[0] / 256)});
+      if (p.tiles.split > 0) S = std::min<int64_t>({(int64_t)p.tiles.split, (int64_t)T6_COL_SMAX, P.pwsize[0]});   // tile knob
       P.colS = (int)S;
       P.colpart = (float*)(w + p.auxi[1]);
       P.colcnt = (unsigned*)(w + p.auxi[1] + al((size_t)T6_COL_SMAX * P.Nc * P.T * 4));

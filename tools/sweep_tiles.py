@@ -54,6 +54,8 @@ def cases():
         ("matmul_f32", lambda: bw("matmul_f32"),
          ["split=1", "split=2", "stages=2", "mode=0", "stages=2,mode=0"]),
         # T6: the streaming scan vs the segmented grid-barrier scan at three segment sizes
+        # T6 MBBS: the column fold's row-range splits (default: fill 8 × 256 threads per SM)
+        ("mbbs_f32", lambda: bw("mbbs_f32"), [f"split={c}" for c in (4, 6, 7, 8, 9, 10, 12, 16, 24, 32)]),
         ("prefix_sum_f32", lambda: bw("prefix_sum_f32"),
          [f"seg={g}" for g in (65536, 262144, 1048576)]),
         ("prl_B", lambda: (S.prl(1 << 14, 1 << 20), G.prl_inputs(1 << 14, 1 << 20)),
@@ -140,7 +142,7 @@ def main():
             # fall back to the template defaults, not to the nearest bucket it was timed with)
             knobs = {"T1_stencil": ("zchunk", "l2pf"), "T2_reduce": ("split",), "T4_tcgen05_contraction": ("bn", "split", "stages"),
                      "T5_prl_pairwise": ("split", "vec", "stages", "bk"), "T3_simt_contraction": ("split",),
-                     "T6_prefix_scan": ("seg",)}.get(d["template"], ())
+                     "T6_prefix_scan": ("seg", "split")}.get(d["template"], ())
             tiles = {k: int(d["tiles"][k]) for k in knobs if k in d["tiles"]}
         fname = spec["f"]
         opcls = next((o for o in spec["ops"] if o == "PS_ADD"), None) or next((o for o in spec["ops"] if o != "CC"), "CC")
