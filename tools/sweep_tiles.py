@@ -46,7 +46,7 @@ def cases():
          + ["zchunk=8,l2pf=2", "zchunk=8,l2pf=1", "zchunk=16,l2pf=2", "zchunk=8,vec=8",
             "zchunk=8,stages=3", "zchunk=16,stages=6"]),
         ("gaussian2d", lambda: bw("gaussian2d"),
-         [f"zchunk={z}" for z in (8, 16, 32, 64)]),
+         [f"zchunk={z}" for z in (8, 12, 16, 20, 24, 32, 48, 64)] + ["zchunk=16,mode=1", "zchunk=32,mode=1"]),
         # T5: records per thread (vec = R), CTAs per SM (stages), DB-loop unroll (bk), split
         ("prl_A", lambda: bw("prl_A"),
          ["split=1", "vec=8", "stages=2", "bk=2", "bk=8", "vec=8,bk=2"]),
