@@ -9,7 +9,7 @@
 //
 //  * Long unit-stride rows read straight from the input (no pw dims, f = IDENTITY) — the
 //    prefix sum of 2^26 fp32 — take ONE persistent streaming kernel (t6_stream_scan_kernel,
-//    the default): one CTA per SM owns a slice of every segment, brought into a shared-
+//    the default): two CTAs per SM each own a slice of every segment, brought into a shared-
 //    memory ring by TMA bulk copies issued three jobs ahead; each CTA publishes its slice
 //    total as a self-validating (tag, value) word, and its exclusive prefix is the carry
 //    plus the totals of the lower CTAs in CTA order (polled by warp 0, no grid barrier);
@@ -676,7 +676,7 @@ __global__ void __launch_bounds__(T6S_THREADS, 3) t6_seg_scan_kernel(const __gri
 // poll finds the other CTAs' totals already published; (C) in-place sequential scan of each
 // thread's K elements from (prefix + its exclusive offset), proxy fence, one bulk store to
 // the output.  HBM: one read + one write per element; deterministic (fixed association).
-constexpr int T6T_THREADS = 512, T6T_NBUF = 4;
+constexpr int T6T_THREADS = 256, T6T_NBUF = 4;   // EXPERIMENT: two CTAs per SM
 template <class V> struct T6K { static constexpr int K = sizeof(V) == 4 ? 27 : 13; };
 template <class V> constexpr int t6_w() { return T6T_THREADS * T6K<V>::K; }
 template <class V> constexpr int t6_smem() { return T6T_NBUF * t6_w<V>() * (int)sizeof(V) + 128; }
@@ -721,12 +721,12 @@ __device__ __forceinline__ bool t6_read(const unsigned long long* slot, unsigned
 
 // Warp 0: (Σ_{i<G} prev[i], Σ_{i<b} cur[i]) once their tags match — lane-strided
 // sequential sums, then a fixed shuffle tree (deterministic for a given G, b); all the
-// reads of a lane are issued together (G ≤ 256: 8 per lane and slot)
+// reads of a lane are issued together (G ≤ 320: 10 per lane and slot)
 template <class V>
 __device__ __forceinline__ void t6_sums_tagged(const unsigned long long* pw, unsigned ptag, bool want_prev,
                                                const unsigned long long* cw, unsigned ctag, int G, int b,
                                                V* all_prev, V* lower) {
-  constexpr int R = 8, S = sizeof(V) == 4 ? 1 : 2;
+  constexpr int R = 10, S = sizeof(V) == 4 ? 1 : 2;
   const int lane = threadIdx.x;
   bool okp[R], okc[R];
   V vp[R], vc[R];
@@ -767,7 +767,7 @@ __device__ __forceinline__ void t6_sums_tagged(const unsigned long long* pw, uns
 }
 
 template <class V>
-__global__ void __launch_bounds__(T6T_THREADS, 1) t6_stream_scan_kernel(const __grid_constant__ T6Params P) {
+__global__ void __launch_bounds__(T6T_THREADS, 2) t6_stream_scan_kernel(const __grid_constant__ T6Params P) {
   constexpr int K = T6K<V>::K, W = t6_w<V>(), VEC = 16 / sizeof(V), NB = T6T_NBUF;
   extern __shared__ __align__(128) uint8_t t6_dyn[];
   V* buf = reinterpret_cast<V*>(t6_dyn);                            // [NB][W] (stays in the shared window)
@@ -973,7 +973,7 @@ mdh_status prepare_t6(Plan* p) {
   }
   if (seg) {                              // streaming scan (default)
     p->auxi.assign(1, -1);
-    p->ws_kernel = 256 + al((size_t)8 * 256 * 16);     // header, 8 × G tagged totals
+    p->ws_kernel = 256 + al((size_t)8 * 320 * 16);     // header, 8 × G tagged totals
     return MDH_OK;
   }
   p->auxi.clear();
@@ -1026,7 +1026,12 @@ static mdh_status launch_stream(T6Params& P, cudaStream_t st) {
   int dev = 0, sms = 148;
   MDH_CUDA(cudaGetDevice(&dev));
   MDH_CUDA(cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev));
-  const int G = std::min(sms, 256);       // one CTA per SM; ≤ 256 (8 tags per lane when polling)
+  static int per = 0;                     // resident CTAs per SM (2 for every value type)
+  if (per == 0) {
+    MDH_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per, t6_stream_scan_kernel<V>, T6T_THREADS, t6_smem<V>()));
+    per = std::max(1, std::min(per, 2));
+  }
+  const int G = std::min(per * sms, 320);  // co-resident (cooperative launch); ≤ 320: 10 tags per polling lane
   void* args[] = {&P};
   MDH_CUDA(cudaLaunchCooperativeKernel((const void*)t6_stream_scan_kernel<V>, dim3(G), dim3(T6T_THREADS), args,
                                        t6_smem<V>(), st));
